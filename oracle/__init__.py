@@ -1,0 +1,229 @@
+"""CPU oracle for the Speculative Reconvergence hot path -- TEST INFRASTRUCTURE.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
+``--impl reference`` legs may import this package.  The product path
+(``paper_conf_cgo_damanijskymg20_b200``) never imports it, and this package
+never imports the product path.  See ``oracle/oracle.h`` for what each
+function computes and which paper passage it follows.
+
+This module is argument marshalling only (ctypes + numpy); every number is
+computed by the plain C in ``oracle/*.c``.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB = os.path.join(HERE, "liboracle.so")
+SOURCES = ["philox.c", "srmath.c", "divloop.c", "commoncall.c", "mcml.c", "warpsim.c",
+           "pathtrace.c"]
+CFLAGS = ["-O2", "-std=gnu11", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
+          "-Wall", "-Wno-unused-function"]
+
+TAG_DIV, TAG_CALL, TAG_MC, TAG_PT = 1, 2, 3, 4
+PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
+# region ids (oracle.h)
+DL = dict(ENTRY=0, PROLOG=1, EXPENSIVE=2, EPILOG=3, ROUND=4, RELEASE=5, ADVANCE=6)
+CC = dict(ENTRY=0, THEN=1, ELSE_PRE=2, CALL=3, ELSE_POST=4, MERGE=5)
+LM = dict(ENTRY=0, LAUNCH=1, STEP=2, STEP_BOUNDARY=3, STEP_INTERACT=4, ROUND=5, RELEASE=6,
+          ADVANCE=7)
+MC_COUNTERS = ["photons", "steps", "rd_exits", "tt_exits", "rr_kills", "rr_survive", "capped",
+               "zero_w"]
+MAX_LAYERS = 8
+
+
+def build(force: bool = False) -> str:
+    srcs = [os.path.join(HERE, s) for s in SOURCES if os.path.exists(os.path.join(HERE, s))]
+    newest = max(os.path.getmtime(s) for s in srcs + [os.path.join(HERE, "oracle.h")])
+    if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < newest:
+        tmp = LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, *srcs, "-lm"])
+        os.replace(tmp, LIB)
+    return LIB
+
+
+class _Layer(C.Structure):
+    _fields_ = [("n", C.c_float), ("mua", C.c_float), ("mus", C.c_float), ("g", C.c_float),
+                ("d", C.c_float)]
+
+
+class MCParams(C.Structure):
+    _fields_ = [("n_layers", C.c_uint32), ("layer", _Layer * MAX_LAYERS), ("n_above", C.c_float),
+                ("n_below", C.c_float), ("dr", C.c_float), ("dz", C.c_float), ("nr", C.c_uint32),
+                ("nz", C.c_uint32), ("step_cap", C.c_uint32)]
+
+
+class WsCounts(C.Structure):
+    _fields_ = [("rounds", C.c_uint64), ("execs", C.c_uint64 * 16), ("lanes", C.c_uint64 * 16)]
+
+    def as_dict(self, names):
+        return {"rounds": int(self.rounds),
+                **{k: (int(self.execs[v]), int(self.lanes[v])) for k, v in names.items()}}
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        _lib = C.CDLL(build())
+        L = _lib
+        u32p, u64p, f32p, u8p = (C.POINTER(C.c_uint32), C.POINTER(C.c_uint64),
+                                 C.POINTER(C.c_float), C.POINTER(C.c_uint8))
+        L.or_philox4x32_10.argtypes = [u32p, u32p, u32p]
+        L.or_u01.argtypes = [C.c_uint32]; L.or_u01.restype = C.c_float
+        L.or_u01c.argtypes = [C.c_uint32]; L.or_u01c.restype = C.c_float
+        L.or_sr_logf.argtypes = [C.c_float]; L.or_sr_logf.restype = C.c_float
+        L.or_sr_sincos2pif.argtypes = [C.c_float, f32p, f32p]
+        L.or_sweep_logf_ulp.restype = C.c_double
+        L.or_sweep_sincos2pif_ulp.restype = C.c_double
+        L.or_expensive.argtypes = [C.c_float, C.c_uint32]; L.or_expensive.restype = C.c_float
+        L.or_divloop.argtypes = [u32p, C.c_uint64, C.c_uint64, C.c_uint32, C.c_uint64, f32p, u32p]
+        L.or_divloop_wants.argtypes = [u32p, C.c_uint64, C.c_uint64, C.c_uint32, C.c_uint64, u8p]
+        L.or_commoncall.argtypes = [u32p, C.c_uint64, C.c_uint64, C.c_uint32, C.c_uint64, f32p,
+                                    u8p]
+        L.or_mcml.argtypes = [C.POINTER(MCParams), C.c_uint64, C.c_uint64, C.c_uint64, u64p, u64p,
+                              u64p, u64p, u32p]
+        L.or_mcml_events.argtypes = [C.POINTER(MCParams), C.c_uint64, C.c_uint64, u8p, C.c_uint32]
+        L.or_mcml_events.restype = C.c_uint32
+        L.or_mcml_rsp.argtypes = [C.POINTER(MCParams)]; L.or_mcml_rsp.restype = C.c_float
+        L.ws_divloop.argtypes = [u8p, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int, C.c_uint32,
+                                 C.POINTER(WsCounts)]
+        L.ws_commoncall.argtypes = [u8p, C.c_uint32, C.c_uint32, C.c_int, C.POINTER(WsCounts)]
+        L.ws_loopmerge.argtypes = [u32p, u8p, u64p, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int,
+                                   C.c_uint32, C.POINTER(WsCounts)]
+        L.ws_divloop_optimum.argtypes = [u8p, C.c_uint32, C.c_uint32]
+        L.ws_divloop_optimum.restype = C.c_uint32
+        if hasattr(L, "or_pt_render"):
+            _bind_pt(L)
+    return _lib
+
+
+def _p(a, ct):
+    return a.ctypes.data_as(C.POINTER(ct))
+
+
+# ---------------------------------------------------------------- RNG / math
+def philox(ctr, key):
+    c = np.asarray(ctr, dtype=np.uint32); k = np.asarray(key, dtype=np.uint32)
+    out = np.zeros(4, np.uint32)
+    lib().or_philox4x32_10(_p(c, C.c_uint32), _p(k, C.c_uint32), _p(out, C.c_uint32))
+    return out
+
+
+def sr_logf(x: float) -> float:
+    return lib().or_sr_logf(x)
+
+
+def sr_sincos2pif(x: float):
+    s, c = C.c_float(), C.c_float()
+    lib().or_sr_sincos2pif(x, C.byref(s), C.byref(c))
+    return s.value, c.value
+
+
+# ---------------------------------------------------------------- config 1
+def divloop(t0, n, iters, seed, p_u32=1 << 29, fma_count=1000):
+    prm = np.array([p_u32, fma_count], np.uint32)
+    acc = np.zeros(n, np.float32); cnt = np.zeros(n, np.uint32)
+    lib().or_divloop(_p(prm, C.c_uint32), t0, n, iters, seed, _p(acc, C.c_float),
+                     _p(cnt, C.c_uint32))
+    return acc, cnt
+
+
+def divloop_wants(t0, n, iters, seed, p_u32=1 << 29, fma_count=1000):
+    prm = np.array([p_u32, fma_count], np.uint32)
+    w = np.zeros(n * iters, np.uint8)
+    lib().or_divloop_wants(_p(prm, C.c_uint32), t0, n, iters, seed, _p(w, C.c_uint8))
+    return w.reshape(n, iters)
+
+
+# ---------------------------------------------------------------- config 2
+def commoncall(t0, n, iters, seed, split_u32=1 << 31, fma_count=2000):
+    prm = np.array([fma_count, split_u32], np.uint32)
+    y = np.zeros(n, np.float32); arm = np.zeros(n, np.uint8)
+    lib().or_commoncall(_p(prm, C.c_uint32), t0, n, iters, seed, _p(y, C.c_float),
+                        _p(arm, C.c_uint8))
+    return y, arm
+
+
+# ---------------------------------------------------------------- configs 3/5
+def mc_params(layers, n_above=1.0, n_below=1.0, dr=0.01, dz=0.002, nr=256, nz=255,
+              step_cap=100000) -> MCParams:
+    p = MCParams()
+    p.n_layers = len(layers)
+    for i, (n_, mua, mus, g, d) in enumerate(layers):
+        p.layer[i] = _Layer(n_, mua, mus, g, d)
+    p.n_above, p.n_below, p.dr, p.dz = n_above, n_below, dr, dz
+    p.nr, p.nz, p.step_cap = nr, nz, step_cap
+    return p
+
+
+def mcml(p: MCParams, id0, count, seed, steps=False):
+    A = np.zeros(p.nz * p.nr, np.uint64); Rd = np.zeros(p.nr, np.uint64)
+    Tt = np.zeros(p.nr, np.uint64); cnt = np.zeros(8, np.uint64)
+    st = np.zeros(count, np.uint32) if steps else None
+    lib().or_mcml(C.byref(p), id0, count, seed, _p(A, C.c_uint64), _p(Rd, C.c_uint64),
+                  _p(Tt, C.c_uint64), _p(cnt, C.c_uint64),
+                  _p(st, C.c_uint32) if steps else None)
+    out = dict(A=A.reshape(p.nz, p.nr), Rd=Rd, Tt=Tt, counters=dict(zip(MC_COUNTERS, map(int, cnt))),
+               counters_raw=cnt)
+    if steps:
+        out["steps"] = st
+    return out
+
+
+def mcml_events(p: MCParams, pid, seed, cap=1 << 20):
+    ev = np.zeros(cap, np.uint8)
+    n = lib().or_mcml_events(C.byref(p), pid, seed, _p(ev, C.c_uint8), cap)
+    return ev[:n].copy()
+
+
+def mcml_rsp(p: MCParams) -> float:
+    return lib().or_mcml_rsp(C.byref(p))
+
+
+# ---------------------------------------------------------------- simulator
+def ws_divloop(want, mode, T, W=32, n_valid=None):
+    want = np.ascontiguousarray(want, np.uint8)
+    n_valid = want.shape[0] if n_valid is None else n_valid
+    o = WsCounts()
+    lib().ws_divloop(_p(want, C.c_uint8), W, n_valid, want.shape[1], mode, T, C.byref(o))
+    return o.as_dict(DL)
+
+
+def ws_commoncall(arm, mode, W=32):
+    arm = np.ascontiguousarray(arm, np.uint8)
+    o = WsCounts()
+    lib().ws_commoncall(_p(arm, C.c_uint8), W, arm.shape[0], mode, C.byref(o))
+    return o.as_dict(CC)
+
+
+def ws_loopmerge(nsteps, mode, T, W=32, events=None):
+    """nsteps: [n_valid, K] uint32; events: optional list-of-lists of uint8 arrays."""
+    nsteps = np.ascontiguousarray(nsteps, np.uint32)
+    n_valid, K = nsteps.shape
+    o = WsCounts()
+    if events is not None:
+        flat = [events[l][k] for l in range(n_valid) for k in range(K)]
+        off = np.zeros(len(flat), np.uint64)
+        np.cumsum([len(e) for e in flat[:-1]], out=off[1:]) if len(flat) > 1 else None
+        ev = np.ascontiguousarray(np.concatenate(flat) if flat else np.zeros(1), np.uint8)
+        lib().ws_loopmerge(_p(nsteps, C.c_uint32), _p(ev, C.c_uint8), _p(off, C.c_uint64), W,
+                           n_valid, K, mode, T, C.byref(o))
+    else:
+        lib().ws_loopmerge(_p(nsteps, C.c_uint32), None, None, W, n_valid, K, mode, T, C.byref(o))
+    return o.as_dict(LM)
+
+
+def ws_divloop_optimum(want):
+    want = np.ascontiguousarray(want, np.uint8)
+    return lib().ws_divloop_optimum(_p(want, C.c_uint8), want.shape[0], want.shape[1])
+
+
+def _bind_pt(L):  # filled in by pathtrace support
+    pass

@@ -1,0 +1,132 @@
+/*
+ * oracle.h -- CPU ORACLE for the Speculative Reconvergence hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+ * cpu_baseline / --impl reference legs of bench.py may load liboracle.so.
+ * The product path (libsr.so, paper_conf_cgo_damanijskymg20_b200/) never
+ * includes, links or calls anything in this directory, and nothing here
+ * includes or links the CUDA path.  The two share no code.
+ *
+ * Paper: Damani et al., "Speculative Reconvergence for Improved SIMT
+ * Efficiency", CGO'20.  Citations "P:N" are /root/reference/PAPER.md lines.
+ *
+ * Part 1 (divloop.c, commoncall.c, mcml.c, pathtrace.c): the unannotated
+ *   program of Fig. 2 / Listing 1 executed one task
+ *   at a time.  Convergence barriers "are not required for correctness of the
+ *   program", so this is the expected output of EVERY mode,
+ *   threshold, block size and GPU count.
+ * Part 2 (warpsim.c): a lane-mask warp simulator that executes the PDOM
+ *   rule and the Speculative Reconvergence rule with a
+ *   soft-barrier threshold (Sec. 4.6) over per-lane event
+ *   streams produced by part 1, and counts region executions / active lanes.
+ *
+ * Parity status per function is listed in DESIGN.md ("Oracle pins").
+ * Built with: gcc -O2 -std=c11 -ffp-contract=off -fno-fast-math -fPIC -shared
+ */
+#ifndef SR_ORACLE_H
+#define SR_ORACLE_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- philox.c : Philox4x32-10 counter-based RNG (paper is silent on RNG;
+ * DESIGN.md reading R1).  ctr = {event, (tag<<16)|sub, task_lo, task_hi},
+ * key = {seed_lo, seed_hi}. */
+enum { OR_TAG_DIV = 1, OR_TAG_CALL = 2, OR_TAG_MC = 3, OR_TAG_PT = 4 };
+void or_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out[4]);
+float or_u01(uint32_t u);   /* (u>>8) * 2^-24     in [0,1) */
+float or_u01c(uint32_t u);  /* ((u>>8)+1) * 2^-24 in (0,1] */
+
+/* ---- srmath.c : the two transcendental functions of the MC / PT steps,
+ * defined op-by-op (reading R5) so CPU and GPU round identically. */
+float or_sr_logf(float x);                             /* x in (0, 1]           */
+void  or_sr_sincos2pif(float xi, float* s, float* c);  /* xi = k*2^-24, k<2^24  */
+/* exhaustive accuracy sweeps (all 2^24 RNG-reachable inputs) vs double libm:
+ * returns max |error| in units of the float ulp of the exact result. */
+double or_sweep_logf_ulp(void);
+double or_sweep_sincos2pif_ulp(void);
+
+/* ---- divloop.c : config 1, divergent condition in a loop (Fig. 2(a)). */
+typedef struct { uint32_t p_u32, fma_count; } or_divloop_params;
+/* threads [t0, t0+n): acc[n], cnt[n] */
+void or_divloop(const or_divloop_params* p, uint64_t t0, uint64_t n, uint32_t iters,
+                uint64_t seed, float* acc, uint32_t* cnt);
+/* event stream for the simulator: want[(t-t0)*iters + i] in {0,1} */
+void or_divloop_wants(const or_divloop_params* p, uint64_t t0, uint64_t n, uint32_t iters,
+                      uint64_t seed, uint8_t* want);
+float or_expensive(float u, uint32_t fma_count);  /* the common code of c3/c4 */
+
+/* ---- commoncall.c : config 2, common function call (Fig. 2(c)). */
+typedef struct { uint32_t fma_count, split_u32; } or_commoncall_params;
+void or_commoncall(const or_commoncall_params* p, uint64_t t0, uint64_t n, uint32_t iters,
+                   uint64_t seed, float* y, uint8_t* arm /* may be NULL: arm of iter 0 */);
+
+/* ---- mcml.c : configs 3/5, MCML photon transport in a layered slab. */
+#define OR_MC_MAX_LAYERS 8
+typedef struct { float n, mua, mus, g, d; } or_layer;  /* cm^-1, cm */
+typedef struct {
+  uint32_t n_layers;
+  or_layer layer[OR_MC_MAX_LAYERS];
+  float n_above, n_below;
+  float dr, dz;
+  uint32_t nr, nz;
+  uint32_t step_cap;
+} or_mcml_params;
+/* counter slots (u64) */
+enum { OR_MC_PHOTONS = 0, OR_MC_STEPS, OR_MC_RD_EXITS, OR_MC_TT_EXITS, OR_MC_RR_KILLS,
+       OR_MC_RR_SURVIVE, OR_MC_CAPPED, OR_MC_ZERO_W, OR_MC_NCOUNTERS = 8 };
+/* Adds into caller-zeroed tallies: A[nz*nr] (iz-major), Rd[nr], Tt[nr],
+ * cnt[OR_MC_NCOUNTERS].  Photon ids [id0, id0+count).  steps_out (may be
+ * NULL) receives the per-photon step count. */
+void or_mcml(const or_mcml_params* p, uint64_t id0, uint64_t count, uint64_t seed,
+             uint64_t* A, uint64_t* Rd, uint64_t* Tt, uint64_t* cnt, uint32_t* steps_out);
+/* Per-photon event stream for the simulator (one byte per step):
+ * bit0 = boundary (else interaction).  Returns number of steps written
+ * (<= cap); stops at cap. */
+uint32_t or_mcml_events(const or_mcml_params* p, uint64_t id, uint64_t seed,
+                        uint8_t* ev, uint32_t cap);
+/* MCML Fresnel reflectance (all-or-none decision uses it) */
+float or_mcml_fresnel(float ni, float nt, float ca1, float* ca2);
+/* Rsp as defined in mcml.c (specular reflectance at launch) */
+float or_mcml_rsp(const or_mcml_params* p);
+
+/* ---- warpsim.c : lane-mask warp simulator (oracle part 2). */
+enum { WS_PDOM = 0, WS_SPEC_LOOP = 1, WS_SPEC_CALL = 2 };
+/* regions of the divloop program (Listing 1) */
+enum { WS_DL_ENTRY = 0, WS_DL_PROLOG, WS_DL_EXPENSIVE, WS_DL_EPILOG, WS_DL_ROUND,
+       WS_DL_RELEASE, WS_DL_ADVANCE, WS_DL_NREG };
+/* regions of the commoncall program (Fig. 2(c)) */
+enum { WS_CC_ENTRY = 0, WS_CC_THEN, WS_CC_ELSE_PRE, WS_CC_CALL, WS_CC_ELSE_POST,
+       WS_CC_MERGE, WS_CC_NREG };
+/* regions of the loop-merge program (Fig. 2(b), Fig. 3) */
+enum { WS_LM_ENTRY = 0, WS_LM_LAUNCH, WS_LM_STEP, WS_LM_STEP_BOUNDARY,
+       WS_LM_STEP_INTERACT, WS_LM_ROUND, WS_LM_RELEASE, WS_LM_ADVANCE, WS_LM_NREG };
+#define WS_MAX_REG 16
+typedef struct {
+  uint64_t rounds;                 /* SR scheduler rounds (0 under PDOM) */
+  uint64_t execs[WS_MAX_REG];      /* warp-level executions of a region  */
+  uint64_t lanes[WS_MAX_REG];      /* sum of popc(mask) over executions  */
+} ws_counts;
+/* One warp of W<=32 lanes, lane l valid iff l < n_valid.
+ * want[l*L + i] = lane l takes the branch in iteration i. */
+void ws_divloop(const uint8_t* want, uint32_t W, uint32_t n_valid, uint32_t L,
+                int mode, uint32_t T, ws_counts* out);
+/* arm[l] = 1 if lane l takes the then-arm (Fig. 2(c) line 8) */
+void ws_commoncall(const uint8_t* arm, uint32_t W, uint32_t n_valid, int mode, ws_counts* out);
+/* Loop merge: lane l owns tasks k < K; task (l,k) runs nsteps[l*K+k] >= 1 inner
+ * iterations; ev (may be NULL) gives each step's bit0 = boundary, laid out
+ * per task at ev_off[l*K+k]. */
+void ws_loopmerge(const uint32_t* nsteps, const uint8_t* ev, const uint64_t* ev_off,
+                  uint32_t W, uint32_t n_valid, uint32_t K, int mode, uint32_t T,
+                  ws_counts* out);
+/* Exhaustive search (tiny warps) of the minimum number of Expensive
+ * executions over ALL legal interleavings of the iteration-delay program
+ * (any parked subset may be released, any free lane may advance). */
+uint32_t ws_divloop_optimum(const uint8_t* want, uint32_t W, uint32_t L);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,245 @@
+/*
+ * warpsim.c -- ORACLE part 2 (test infrastructure; see oracle.h).
+ *
+ * A lane-mask warp simulator.  It replays the per-lane event streams that
+ * oracle part 1 produces (which iterations want Expensive(), which arm each
+ * lane takes, how many inner steps each task runs) under two convergence
+ * rules and counts, per source region, warp-level executions and active
+ * lanes.  SIMT efficiency, "the average percentage of active threads per
+ * warp", follows from these counts and a per-region instruction
+ * cost table (tools/sass_regions.py reads it off the built cubin).
+ *
+ * PDOM rule (Fig. 1(a)): control follows the
+ * program; a diverged warp reconverges at the immediate post-dominator, so a
+ * region executes once per distinct arrival with mask = the lanes that
+ * reached it.
+ *
+ * Speculative Reconvergence rule (Fig. 1(b), Iteration Delay
+ * P:303-324, Loop Merge P:325-377, soft barrier Sec. 4.6 P:1108-1142,
+ * Fig. 6), one scheduler round at a time:
+ *   P = lanes waiting at the reconvergence point L1 ("Join"ed and arrived),
+ *   R = lanes that can still make progress toward L1 without it.
+ *   P = R = {}          -> exit.
+ *   |P| >= T or R = {}  -> release: all of P run the common code together
+ *                          (all waiting lanes, not T of them: P:1135-1137);
+ *                          R = {} is the "threshold not satisfiable" exit of
+ *                          P:1139-1141.
+ *   otherwise           -> advance: R runs one step of the non-common code
+ *                          (run-ahead of one iteration per round, reading Q5).
+ * The GPU kernels implement the same rule with __ballot_sync; DESIGN.md
+ * readings Q1-Q5, Q11.
+ */
+#include <stdlib.h>
+#include <string.h>
+#include "oracle.h"
+
+static void hit(ws_counts* o, int r, uint32_t mask) {
+  if (!mask) return;
+  o->execs[r] += 1;
+  o->lanes[r] += (uint64_t)__builtin_popcount(mask);
+}
+
+/* ------------------------------------------------------------------ */
+/* Iteration Delay: Fig. 2(a) / Listing 1.                              */
+void ws_divloop(const uint8_t* want, uint32_t W, uint32_t n_valid, uint32_t L, int mode,
+                uint32_t T, ws_counts* o) {
+  memset(o, 0, sizeof *o);
+  if (n_valid > W) n_valid = W;
+  uint32_t valid = n_valid >= 32 ? 0xffffffffu : ((1u << n_valid) - 1u);
+  hit(o, WS_DL_ENTRY, valid);
+  if (mode == WS_PDOM) {
+    for (uint32_t i = 0; i < L; ++i) {
+      hit(o, WS_DL_PROLOG, valid);
+      uint32_t m = 0;
+      for (uint32_t l = 0; l < n_valid; ++l)
+        if (want[l * L + i]) m |= 1u << l;
+      hit(o, WS_DL_EXPENSIVE, m);   /* then-block with the wanting lanes */
+      hit(o, WS_DL_EPILOG, valid);  /* reconverged at the IPDOM */
+    }
+    return;
+  }
+  if (T == 0 || T > 32) T = 32;
+  uint32_t it[32] = {0};
+  uint32_t parked = 0;
+  for (;;) {
+    uint32_t P = parked, R = 0;
+    for (uint32_t l = 0; l < n_valid; ++l)
+      if (!(parked >> l & 1u) && it[l] < L) R |= 1u << l;
+    if (!P && !R) break;
+    o->rounds += 1;
+    hit(o, WS_DL_ROUND, valid);
+    if ((uint32_t)__builtin_popcount(P) >= T || !R) {
+      hit(o, WS_DL_RELEASE, P);
+      hit(o, WS_DL_EXPENSIVE, P);
+      hit(o, WS_DL_EPILOG, P);
+      for (uint32_t l = 0; l < n_valid; ++l)
+        if (P >> l & 1u) it[l] += 1;
+      parked = 0;
+    } else {
+      hit(o, WS_DL_ADVANCE, R);
+      hit(o, WS_DL_PROLOG, R);
+      uint32_t E = 0;
+      for (uint32_t l = 0; l < n_valid; ++l) {
+        if (!(R >> l & 1u)) continue;
+        if (want[l * L + it[l]]) parked |= 1u << l;   /* Join + Wait at L1 */
+        else { E |= 1u << l; it[l] += 1; }             /* run ahead */
+      }
+      hit(o, WS_DL_EPILOG, E);
+    }
+  }
+}
+
+/* ------------------------------------------------------------------ */
+/* Common function call: Fig. 2(c), Sec. 4.4.                          */
+void ws_commoncall(const uint8_t* arm, uint32_t W, uint32_t n_valid, int mode, ws_counts* o) {
+  memset(o, 0, sizeof *o);
+  if (n_valid > W) n_valid = W;
+  uint32_t valid = n_valid >= 32 ? 0xffffffffu : ((1u << n_valid) - 1u);
+  uint32_t then_m = 0;
+  for (uint32_t l = 0; l < n_valid; ++l)
+    if (arm[l]) then_m |= 1u << l;
+  uint32_t else_m = valid & ~then_m;
+  hit(o, WS_CC_ENTRY, valid);
+  if (mode == WS_SPEC_CALL) {
+    hit(o, WS_CC_THEN, then_m);
+    hit(o, WS_CC_ELSE_PRE, else_m);
+    hit(o, WS_CC_CALL, valid);       /* one call, all lanes: reconverged at foo entry */
+    hit(o, WS_CC_ELSE_POST, else_m);
+  } else {
+    hit(o, WS_CC_THEN, then_m);
+    hit(o, WS_CC_CALL, then_m);      /* call site 1 */
+    hit(o, WS_CC_ELSE_PRE, else_m);
+    hit(o, WS_CC_CALL, else_m);      /* call site 2 */
+    hit(o, WS_CC_ELSE_POST, else_m);
+  }
+  hit(o, WS_CC_MERGE, valid);
+}
+
+/* ------------------------------------------------------------------ */
+/* Loop Merge: Fig. 2(b), Fig. 3.                */
+static uint32_t step_mask_split(const uint8_t* ev, const uint64_t* ev_off, uint32_t K,
+                                const uint32_t* kk, const uint32_t* jj, uint32_t mask) {
+  uint32_t b = 0;
+  for (uint32_t l = 0; l < 32; ++l)
+    if (mask >> l & 1u)
+      if (ev[ev_off[l * K + kk[l]] + jj[l]] & 1u) b |= 1u << l;
+  return b;
+}
+
+void ws_loopmerge(const uint32_t* nsteps, const uint8_t* ev, const uint64_t* ev_off, uint32_t W,
+                  uint32_t n_valid, uint32_t K, int mode, uint32_t T, ws_counts* o) {
+  memset(o, 0, sizeof *o);
+  if (n_valid > W) n_valid = W;
+  uint32_t valid = n_valid >= 32 ? 0xffffffffu : ((1u << n_valid) - 1u);
+  uint32_t kk[32] = {0}, jj[32] = {0};
+  hit(o, WS_LM_ENTRY, valid);
+  if (mode == WS_PDOM) {
+    for (uint32_t k = 0; k < K; ++k) {
+      hit(o, WS_LM_LAUNCH, valid);
+      for (uint32_t l = 0; l < n_valid; ++l) { kk[l] = k; jj[l] = 0; }
+      for (;;) {
+        uint32_t m = 0;
+        for (uint32_t l = 0; l < n_valid; ++l)
+          if (jj[l] < nsteps[l * K + k]) m |= 1u << l;
+        if (!m) break;
+        hit(o, WS_LM_STEP, m);
+        if (ev) {
+          uint32_t b = step_mask_split(ev, ev_off, K, kk, jj, m);
+          hit(o, WS_LM_STEP_BOUNDARY, b);
+          hit(o, WS_LM_STEP_INTERACT, m & ~b);
+        }
+        for (uint32_t l = 0; l < n_valid; ++l)
+          if (m >> l & 1u) jj[l] += 1;
+      }
+    }
+    return;
+  }
+  if (T == 0 || T > 32) T = 32;
+  uint32_t alive = 0;
+  uint32_t next[32] = {0};  /* next task index to launch */
+  for (;;) {
+    uint32_t P = alive, R = 0;
+    for (uint32_t l = 0; l < n_valid; ++l)
+      if (!(alive >> l & 1u) && next[l] < K) R |= 1u << l;
+    if (!P && !R) break;
+    o->rounds += 1;
+    hit(o, WS_LM_ROUND, valid);
+    if ((uint32_t)__builtin_popcount(P) >= T || !R) {
+      hit(o, WS_LM_RELEASE, P);
+      hit(o, WS_LM_STEP, P);
+      if (ev) {
+        uint32_t b = step_mask_split(ev, ev_off, K, kk, jj, P);
+        hit(o, WS_LM_STEP_BOUNDARY, b);
+        hit(o, WS_LM_STEP_INTERACT, P & ~b);
+      }
+      for (uint32_t l = 0; l < n_valid; ++l) {
+        if (!(P >> l & 1u)) continue;
+        jj[l] += 1;
+        if (jj[l] == nsteps[l * K + kk[l]]) alive &= ~(1u << l);
+      }
+    } else {
+      hit(o, WS_LM_ADVANCE, R);
+      hit(o, WS_LM_LAUNCH, R);   /* epilog of the finished task + prolog of the next */
+      for (uint32_t l = 0; l < n_valid; ++l) {
+        if (!(R >> l & 1u)) continue;
+        kk[l] = next[l]++;
+        jj[l] = 0;
+        alive |= 1u << l;
+      }
+    }
+  }
+}
+
+/* ------------------------------------------------------------------ */
+/* Exhaustive optimum of the iteration-delay program for W <= 4, L <= 4:
+ * 0-1 BFS over (it[l], parked[l]); advancing one free lane costs 0,
+ * releasing any non-empty subset of parked lanes costs 1 Expensive execution. */
+uint32_t ws_divloop_optimum(const uint8_t* want, uint32_t W, uint32_t L) {
+  if (W == 0 || W > 4 || L > 4) return 0xffffffffu;
+  uint32_t base = L + 1u;
+  uint32_t nstate = 1;
+  for (uint32_t l = 0; l < W; ++l) nstate *= base * 2u;
+  uint32_t* dist = (uint32_t*)malloc(sizeof(uint32_t) * nstate);
+  /* 0-1 BFS deque: dist[] of a state improves at most L*W+1 times, so
+   * front pushes <= nstate*32 and back pushes <= nstate*96 */
+  uint32_t* dq = (uint32_t*)malloc(sizeof(uint32_t) * nstate * 128u);
+  for (uint32_t s = 0; s < nstate; ++s) dist[s] = 0xffffffffu;
+  /* state encoding: digit l = it[l]*2 + parked[l] in base 2(L+1) */
+  uint32_t head = nstate * 32u, tail = head;
+  dist[0] = 0;
+  dq[tail++] = 0;
+  uint32_t best = 0xffffffffu;
+  while (head < tail) {
+    uint32_t s = dq[head++];
+    uint32_t d = dist[s];
+    uint32_t it[4], pk[4], x = s;
+    for (uint32_t l = 0; l < W; ++l) { uint32_t dg = x % (2u * base); x /= 2u * base; it[l] = dg / 2u; pk[l] = dg % 2u; }
+    int done = 1;
+    for (uint32_t l = 0; l < W; ++l) if (it[l] < L || pk[l]) done = 0;
+    if (done) { if (d < best) best = d; continue; }
+    /* cost-0 moves: advance one free lane */
+    for (uint32_t l = 0; l < W; ++l) {
+      if (pk[l] || it[l] >= L) continue;
+      uint32_t nit[4], npk[4];
+      memcpy(nit, it, sizeof nit); memcpy(npk, pk, sizeof npk);
+      if (want[l * L + it[l]]) npk[l] = 1; else nit[l] += 1;
+      uint32_t ns = 0, mul = 1;
+      for (uint32_t q = 0; q < W; ++q) { ns += (nit[q] * 2u + npk[q]) * mul; mul *= 2u * base; }
+      if (dist[ns] > d) { dist[ns] = d; dq[--head] = ns; }
+    }
+    /* cost-1 moves: release a non-empty subset of parked lanes */
+    uint32_t pmask = 0;
+    for (uint32_t l = 0; l < W; ++l) if (pk[l]) pmask |= 1u << l;
+    for (uint32_t sub = pmask; sub; sub = (sub - 1u) & pmask) {
+      uint32_t nit[4], npk[4];
+      memcpy(nit, it, sizeof nit); memcpy(npk, pk, sizeof npk);
+      for (uint32_t l = 0; l < W; ++l) if (sub >> l & 1u) { npk[l] = 0; nit[l] += 1; }
+      uint32_t ns = 0, mul = 1;
+      for (uint32_t q = 0; q < W; ++q) { ns += (nit[q] * 2u + npk[q]) * mul; mul *= 2u * base; }
+      if (dist[ns] > d + 1u) { dist[ns] = d + 1u; dq[tail++] = ns; }
+    }
+  }
+  free(dist);
+  free(dq);
+  return best;
+}

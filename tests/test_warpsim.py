@@ -1,0 +1,133 @@
+"""Pins of the lane-mask warp simulator (oracle part 2).
+
+Fig. 1 worked example, closed forms, conservation laws and brute-force
+enumeration of every want pattern / trip-count combination of 4-lane warps,
+plus an exhaustive search over all legal interleavings for the optimum.
+"""
+import itertools
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle import PDOM, SPEC_LOOP, SPEC_CALL
+from paper_conf_cgo_damanijskymg20_b200 import inputs as I
+
+
+def test_fig1_worked_example():
+    # Fig. 1: 4 lanes each want Expensive() in a different iteration.
+    want = np.eye(4, dtype=np.uint8)
+    pd = oracle.ws_divloop(want, PDOM, 0, W=4)
+    assert pd["EXPENSIVE"] == (4, 4)      # run 4x serially, 1 lane each: 25%
+    sr = oracle.ws_divloop(want, SPEC_LOOP, 4, W=4)
+    assert sr["EXPENSIVE"] == (1, 4)      # run once, converged: 100%
+
+
+def _all_patterns(W, L):
+    for bits in range(1 << (W * L)):
+        yield np.array([(bits >> b) & 1 for b in range(W * L)], np.uint8).reshape(W, L)
+
+
+@pytest.mark.parametrize("L", [1, 2, 3, 4])
+def test_divloop_bruteforce_4_lanes(L):
+    W = 4
+    for want in _all_patterns(W, L):
+        K = want.sum(1)
+        pd = oracle.ws_divloop(want, PDOM, 0, W=W)
+        assert pd["EXPENSIVE"][1] == K.sum()
+        assert pd["EXPENSIVE"][0] == int(want.any(0).sum())
+        execs = []
+        for T in range(1, W + 1):
+            sr = oracle.ws_divloop(want, SPEC_LOOP, T, W=W)
+            assert sr["EXPENSIVE"][1] == K.sum()                       # conservation
+            assert sr["EXPENSIVE"][0] >= K.max()                        # lower bound
+            assert sr["PROLOG"][1] == W * L                              # every iteration once
+            execs.append(sr["EXPENSIVE"][0])
+        assert execs[0] == pd["EXPENSIVE"][0]                           # T=1 == PDOM
+        assert execs[-1] == K.max()                                     # T=W: max_l K_l
+
+
+def test_divloop_optimum_exhaustive_search():
+    rng = np.random.default_rng(0)
+    pats = list(_all_patterns(3, 3)) + [rng.integers(0, 2, (4, 4)).astype(np.uint8)
+                                        for _ in range(40)]
+    for want in pats:
+        opt = oracle.ws_divloop_optimum(want)
+        assert opt == want.sum(1).max()
+        assert oracle.ws_divloop(want, SPEC_LOOP, want.shape[0], W=want.shape[0])["EXPENSIVE"][0] == opt
+
+
+def test_divloop_closed_forms_config1():
+    c = I.C1
+    want = oracle.divloop_wants(0, c.n_threads, c.iters, I.PRIMARY_SEED, c.p_u32)
+    p = c.p_u32 / 2**32
+    n_warps = c.n_threads // 32
+    pd, t32, t1 = [], [], []
+    for w in range(n_warps):
+        ww = want[32 * w:32 * w + 32]
+        pd.append(oracle.ws_divloop(ww, PDOM, 0)["EXPENSIVE"][0])
+        s32 = oracle.ws_divloop(ww, SPEC_LOOP, 32)
+        t32.append(s32["EXPENSIVE"][0])
+        assert t32[-1] == ww.sum(1).max()
+        if w < 64:
+            t1.append(oracle.ws_divloop(ww, SPEC_LOOP, 1)["EXPENSIVE"][0])
+            assert t1[-1] == pd[-1]
+    q = 1 - (1 - p) ** 32
+    # PDOM: E[execs per warp] = iters * (1 - (1-p)^32) = 63.108
+    assert abs(np.mean(pd) - c.iters * q) < 5 * math.sqrt(c.iters * q * (1 - q) / n_warps)
+    # SR, T=32: E[max of 32 Binomial(64, p)] = sum_k (1 - F(k)^32) = 13.855
+    from scipy.stats import binom
+    ks = np.arange(0, c.iters + 1)
+    e_max = float(np.sum(1 - binom.cdf(ks, c.iters, p) ** 32))
+    assert abs(e_max - 13.855) < 5e-3
+    assert abs(np.mean(t32) - e_max) < 0.15
+
+
+def test_divloop_partial_warp_and_threshold_above_valid():
+    want = np.array([[1, 0, 1], [0, 1, 1], [1, 1, 0]], np.uint8)
+    sr = oracle.ws_divloop(want, SPEC_LOOP, 32, W=32)   # T > valid lanes: R = {} releases
+    assert sr["EXPENSIVE"] == (2, 6)
+    assert sr["ROUND"][1] == sr["ROUND"][0] * 3          # invalid lanes never in a mask
+
+
+def test_commoncall_counts():
+    for arm in ([1] * 32, [0] * 32, [1, 0] * 16):
+        arm = np.array(arm, np.uint8)
+        pd = oracle.ws_commoncall(arm, PDOM)
+        sc = oracle.ws_commoncall(arm, SPEC_CALL)
+        assert pd["CALL"][0] == int(arm.any()) + int((1 - arm).any())
+        assert pd["CALL"][1] == 32 and sc["CALL"] == (1, 32)
+    # foo-region efficiency 50% -> 100% for the 50/50 split
+    arm = np.array([1, 0] * 16, np.uint8)
+    pd = oracle.ws_commoncall(arm, PDOM)
+    assert pd["CALL"][1] / (32 * pd["CALL"][0]) == 0.5
+
+
+@pytest.mark.parametrize("K", [1, 2])
+def test_loopmerge_bruteforce_4_lanes(K):
+    W = 4
+    for ns in itertools.product(range(1, 5), repeat=W * K):
+        n = np.array(ns, np.uint32).reshape(W, K)
+        pd = oracle.ws_loopmerge(n, PDOM, 0, W=W)
+        assert pd["STEP"][1] == n.sum()
+        assert pd["STEP"][0] == n.max(0).sum()                  # sum_k max_l n(l,k)
+        t1 = oracle.ws_loopmerge(n, SPEC_LOOP, 1, W=W)
+        assert t1["STEP"] == pd["STEP"]                         # T=1 == PDOM
+        tw = oracle.ws_loopmerge(n, SPEC_LOOP, W, W=W)
+        assert tw["STEP"][0] == n.sum(1).max()                  # max_l sum_k n(l,k)
+        assert tw["STEP"][1] == n.sum()
+        assert tw["LAUNCH"][1] == W * K
+        for T in (2, 3):
+            t = oracle.ws_loopmerge(n, SPEC_LOOP, T, W=W)
+            assert t["STEP"][1] == n.sum() and t["STEP"][0] >= n.sum(1).max()
+
+
+def test_loopmerge_event_split_sums_to_step():
+    p = oracle.mc_params(I.C3.layers)
+    K, W = 3, 32
+    ev = [[oracle.mcml_events(p, l + k * W, 1) for k in range(K)] for l in range(W)]
+    n = np.array([[len(e) for e in row] for row in ev], np.uint32)
+    for mode, T in ((PDOM, 0), (SPEC_LOOP, 32), (SPEC_LOOP, 8)):
+        r = oracle.ws_loopmerge(n, mode, T, events=ev)
+        assert r["STEP_BOUNDARY"][1] + r["STEP_INTERACT"][1] == r["STEP"][1] == n.sum()
