@@ -1,0 +1,182 @@
+/*
+ * sr.h -- C ABI of libsr, the B200-native (sm_100a) Speculative
+ * Reconvergence hot path.
+ *
+ * Paper: Damani, Johnson, Stephenson, Keckler, Yan, McKeown, Giroux,
+ * "Speculative Reconvergence for Improved SIMT Efficiency", CGO 2020.
+ * "P:N" = line N of the paper text.
+ *
+ * The paper's user interface is a Predict(label) directive, a label marking
+ * the reconvergence point, a function name for the common-call case and an
+ * optional soft-barrier threshold (Sec. 4.1; Sec. 4.4
+ * P:999-1002; Sec. 4.6).  Here the prediction region and label are
+ * fixed per workload (the annotated loops of Fig. 2) and a call
+ * selects the schedule with `mode` and the soft barrier with `threshold`.
+ *
+ * Conventions for every entry point:
+ *   - returns SR_OK (0) or a negative sr_status; never throws, never aborts;
+ *     sr_last_error() describes the last failure of the calling thread;
+ *   - arguments are validated before any GPU work is enqueued;
+ *   - all GPU work is enqueued on the stream given to sr_init (a cudaStream_t
+ *     passed as void*; NULL = legacy default stream), in order;
+ *   - device memory is owned by the caller; the library allocates none;
+ *   - one process-global context per process (= per GPU); not re-entrant.
+ */
+#ifndef SR_H
+#define SR_H
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define SR_API __attribute__((visibility("default")))
+#else
+#define SR_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  SR_OK = 0,
+  SR_E_INVALID = -1,  /* bad argument (see each call)                       */
+  SR_E_STATE = -2,    /* call before sr_init / after sr_finalize / no run   */
+  SR_E_NOMEM = -3,    /* workspace or destination buffer too small          */
+  SR_E_CUDA = -4      /* CUDA runtime error; message carries the CUDA text  */
+} sr_status;
+
+/* Schedules.  SR_PDOM: plain structured code; the compiler reconverges at
+ * the immediate post-dominator.  SR_SPEC_LOOP:
+ * Iteration Delay / Loop Merge (Fig. 1(b)) with soft barrier
+ * (Sec. 4.6).  SR_SPEC_CALL: reconvergence at the entry of the common
+ * callee (Fig. 2(c), Sec. 4.4). */
+typedef enum { SR_PDOM = 0, SR_SPEC_LOOP = 1, SR_SPEC_CALL = 2 } sr_mode;
+
+typedef enum {
+  SR_WL_DIVLOOP = 0,     /* Fig. 2(a): divergent condition in a loop (config 1) */
+  SR_WL_COMMONCALL = 1,  /* Fig. 2(c): common function call          (config 2) */
+  SR_WL_MCML = 2,        /* Fig. 2(b): MC photon transport, loop merge (3, 5)  */
+  SR_WL_PATHTRACE = 3    /* Fig. 2(b): path tracer, loop merge       (config 4) */
+} sr_workload_kind;
+
+/* sr_workload.flags */
+#define SR_F_SCHED 1u   /* also write per-warp schedule counters (instrumented kernels) */
+#define SR_F_STATIC 2u  /* MCML / PATHTRACE: static task->lane assignment (lane l owns tasks
+                           l + k*n_threads) instead of the default dynamic per-warp claiming.
+                           Results are identical; only the schedule differs. */
+
+#define SR_MAX_LAYERS 8
+typedef struct { float n, mua, mus, g, d; } sr_layer;  /* -, 1/cm, 1/cm, -, cm */
+
+typedef struct {
+  uint32_t p_u32;      /* P(condition) = p_u32 / 2^32 (1/8: 2^29)               */
+  uint32_t fma_count;  /* FMAs in Expensive(); multiple of 8 (1000)             */
+} sr_divloop_params;
+
+typedef struct {
+  uint32_t fma_count;  /* FMAs in the common callee foo(); multiple of 8 (2000)  */
+  uint32_t split_u32;  /* P(then-arm) = split_u32 / 2^32 (1/2: 2^31)             */
+} sr_commoncall_params;
+
+typedef struct {
+  uint32_t n_layers;   /* 1 .. SR_MAX_LAYERS                                     */
+  sr_layer layers[SR_MAX_LAYERS];
+  float n_above, n_below;  /* ambient refractive indices                         */
+  float dr, dz;            /* tally grid spacing, cm                             */
+  uint32_t nr, nz;         /* tally grid size (nr, nz >= 1)                      */
+  uint32_t step_cap;       /* a photon dies after this many steps (>= 1)         */
+} sr_mcml_params;
+
+typedef struct {
+  const void* scene_dev;  /* device pointer to a scene built by sr_scene_build  */
+  uint64_t scene_bytes;
+  uint32_t width, height; /* image; n_threads must equal width*height           */
+  uint32_t max_depth;     /* bounces per path (>= 1)                            */
+} sr_pathtrace_params;
+
+typedef struct {
+  int32_t kind;            /* sr_workload_kind                                   */
+  uint32_t flags;          /* SR_F_*                                             */
+  uint64_t task_offset;    /* global id of this caller's first task (sharding)  */
+  uint32_t block_threads;  /* CTA size, multiple of 32 in [32,1024]; 0 = default */
+  uint32_t grid_ctas;      /* dynamic-claiming kernels: CTAs; 0 = fill the GPU   */
+  sr_divloop_params divloop;
+  sr_commoncall_params commoncall;
+  sr_mcml_params mcml;
+  sr_pathtrace_params pathtrace;
+} sr_workload;
+
+/* Bind the context to a device, a stream and a caller-owned device
+ * workspace.  May be called again to rebind (e.g. a bigger workspace).
+ * SR_E_CUDA if the device cannot be selected (for instance, no GPU). */
+SR_API int sr_init(int device, void* cuda_stream, void* workspace_dev, size_t workspace_bytes);
+
+/* Workspace regions, each 256-byte aligned, in this order:
+ *   SR_T_PERTHREAD  per-task outputs of the last run:
+ *                   DIVLOOP    n_threads x {float acc; uint32 cnt}  (8 B, AoS)
+ *                   COMMONCALL n_threads x float y
+ *                   MCML       none (0 bytes)
+ *                   PATHTRACE  n_threads x float[3] RGB sum over the spp
+ *   SR_T_GRID       MCML: uint64 A[nz][nr], Rd[nr], Tt[nr]  (fixed point, 2^-32)
+ *   SR_T_COUNTERS   uint64[16] workload counters (see sr_counter_names in DESIGN.md)
+ *   SR_T_SCHED      per warp: uint32[8] schedule counters (only with SR_F_SCHED):
+ *                   {rounds, release rounds, common-code lane-executions,
+ *                    advance rounds, prolog lane-executions, 0, 0, 0}
+ *   SR_T_SCRATCH    internal (claim counters)
+ * GRID and COUNTERS are contiguous so a multi-GPU caller can reduce them
+ * in place as int64 (two's-complement addition = uint64 addition mod 2^64). */
+enum { SR_T_PERTHREAD = 0, SR_T_GRID = 1, SR_T_COUNTERS = 2, SR_T_SCHED = 3, SR_T_SCRATCH = 4 };
+SR_API size_t sr_workspace_bytes(const sr_workload* w, uint64_t n_threads);
+SR_API int sr_workspace_region(const sr_workload* w, uint64_t n_threads, int what, size_t* offset,
+                        size_t* bytes);
+
+/* Run the hot path: n_threads logical threads, each executing `iters`
+ * iterations of its outer loop (DIVLOOP: loop trips; COMMONCALL: repetitions;
+ * MCML: photons per thread = thread coarsening P:336-359; PATHTRACE: samples
+ * per pixel).  threshold: soft-barrier size T in [1,32], 0 = 32 ("wait for
+ * all", Fig. 1(b)); ignored for SR_PDOM; must be 0 or 32 for SR_SPEC_CALL.
+ * SR_SPEC_CALL is valid only for COMMONCALL; SR_SPEC_LOOP only for DIVLOOP,
+ * MCML, PATHTRACE.  Zeroes the output regions, then enqueues the kernel(s);
+ * does not synchronize.  Every output bit is a function of (workload params,
+ * seed, task ids) only -- never of mode, threshold, block size, grid size or
+ * GPU count.
+ * Errors: SR_E_STATE before sr_init; SR_E_INVALID (n_threads == 0,
+ * n_threads*iters overflows 2^63, bad threshold/mode/params); SR_E_NOMEM
+ * (workspace smaller than sr_workspace_bytes); SR_E_CUDA (launch failed). */
+SR_API int sr_run(const sr_workload* w, uint64_t n_threads, uint32_t iters, uint64_t seed, int mode,
+           uint32_t threshold);
+
+/* Copy one region of the last run (what = SR_T_*) into dst, host or device
+ * memory (UVA, cudaMemcpyDefault), on the context stream, then synchronize
+ * that stream.  *written (may be NULL) receives the byte count.
+ * SR_E_NOMEM if dst_bytes is smaller than the region. */
+SR_API int sr_tally(int what, void* dst, size_t dst_bytes, size_t* written);
+
+/* Release the context.  Idempotent. */
+SR_API int sr_finalize(void);
+
+/* Thread-local description of the last error; library-owned; valid until
+ * the next call on this thread.  Empty string after success. */
+SR_API const char* sr_last_error(void);
+
+/* Library build identification: "sm_100a <nvcc version> <flags>". */
+SR_API const char* sr_build_info(void);
+
+/* PATHTRACE scene (config 4): build the BVH over a caller-provided triangle
+ * soup on the host and write the device scene image.
+ *   tris       host, n_tris x 9 floats (v0, v1, v2 xyz), caller-owned
+ *   mat        host, n_tris x uint32 material ids (< n_mats)
+ *   mats       host, n_mats x 8 floats {kind, r, g, b, er, eg, eb, ior}
+ *              kind: 0 diffuse, 1 mirror, 2 dielectric, 3 emissive-only
+ *   cam        host, 12 floats {eye xyz, look-at xyz, up xyz, tan(fov/2), 0, 0}
+ *   dst_dev    device buffer of dst_bytes; *needed receives the size.  If
+ *              dst_dev is NULL only *needed is computed.
+ * The BVH is deterministic for a given input. */
+SR_API int sr_scene_build(const float* tris, const uint32_t* mat, uint32_t n_tris, const float* mats,
+                   uint32_t n_mats, const float* cam, void* dst_dev, size_t dst_bytes,
+                   size_t* needed);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,47 @@
+// sr_internal.h -- host-side internals shared by the libsr translation units.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstddef>
+#include <cstdint>
+#include <string>
+
+#include "../../include/sr.h"
+
+namespace sr {
+
+constexpr int kCounters = 16;
+constexpr int kSchedWords = 8;  // uint32 per warp
+
+// Resolved workspace layout of one (workload, n_threads).
+struct Layout {
+  size_t off[5];
+  size_t bytes[5];
+  size_t total;
+};
+Layout layout_of(const sr_workload& w, uint64_t n_threads);
+
+struct LaunchCtx {
+  cudaStream_t stream;
+  char* ws;          // workspace base
+  Layout lay;
+  int sm_count;
+  uint32_t block;    // resolved CTA size
+};
+
+// Each returns a cudaError_t from the launch (cudaGetLastError after it).
+cudaError_t launch_divloop(const LaunchCtx& c, const sr_workload& w, uint64_t n, uint32_t iters,
+                           uint64_t seed, int mode, uint32_t T);
+cudaError_t launch_commoncall(const LaunchCtx& c, const sr_workload& w, uint64_t n,
+                              uint32_t iters, uint64_t seed, int mode);
+cudaError_t launch_mcml(const LaunchCtx& c, const sr_workload& w, uint64_t n, uint32_t iters,
+                        uint64_t seed, int mode, uint32_t T);
+cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t n,
+                             uint32_t iters, uint64_t seed, int mode, uint32_t T);
+
+// Validation of workload-specific parameters; returns "" when fine.
+std::string check_mcml(const sr_mcml_params& p);
+std::string check_pathtrace(const sr_pathtrace_params& p, uint64_t n_threads);
+size_t pathtrace_perthread_bytes(uint64_t n_threads);
+
+}  // namespace sr

@@ -1,0 +1,210 @@
+"""Thin ctypes binding of libsr (include/sr.h) -- argument marshalling only.
+
+Every function named ``sr_*`` here calls the C entry point of the same name
+and raises :class:`SRError` on a negative status.  Device memory, streams and
+process groups come from PyTorch (plumbing); every step of the hot path runs
+in libsr's CUDA kernels.  There is no CPU fallback: :func:`load` raises if
+``libsr.so`` is missing, and ``sr_init`` fails with ``SR_E_CUDA`` without a GPU.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from dataclasses import dataclass
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libsr.so")
+
+SR_OK, SR_E_INVALID, SR_E_STATE, SR_E_NOMEM, SR_E_CUDA = 0, -1, -2, -3, -4
+PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
+WL_DIVLOOP, WL_COMMONCALL, WL_MCML, WL_PATHTRACE = 0, 1, 2, 3
+F_SCHED, F_STATIC = 1, 2
+T_PERTHREAD, T_GRID, T_COUNTERS, T_SCHED, T_SCRATCH = 0, 1, 2, 3, 4
+MAX_LAYERS = 8
+N_COUNTERS = 16
+SCHED_WORDS = 8
+MC_COUNTERS = ["photons", "steps", "rd_exits", "tt_exits", "rr_kills", "rr_survive", "capped",
+               "zero_w"]
+EXPORTS = ["sr_init", "sr_workspace_bytes", "sr_workspace_region", "sr_run", "sr_tally",
+           "sr_finalize", "sr_last_error", "sr_build_info", "sr_scene_build"]
+
+
+class SRError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"libsr status {code}: {msg}")
+        self.code = code
+
+
+class Layer(C.Structure):
+    _fields_ = [("n", C.c_float), ("mua", C.c_float), ("mus", C.c_float), ("g", C.c_float),
+                ("d", C.c_float)]
+
+
+class DivloopParams(C.Structure):
+    _fields_ = [("p_u32", C.c_uint32), ("fma_count", C.c_uint32)]
+
+
+class CommoncallParams(C.Structure):
+    _fields_ = [("fma_count", C.c_uint32), ("split_u32", C.c_uint32)]
+
+
+class MCMLParams(C.Structure):
+    _fields_ = [("n_layers", C.c_uint32), ("layers", Layer * MAX_LAYERS), ("n_above", C.c_float),
+                ("n_below", C.c_float), ("dr", C.c_float), ("dz", C.c_float), ("nr", C.c_uint32),
+                ("nz", C.c_uint32), ("step_cap", C.c_uint32)]
+
+
+class PathtraceParams(C.Structure):
+    _fields_ = [("scene_dev", C.c_void_p), ("scene_bytes", C.c_uint64), ("width", C.c_uint32),
+                ("height", C.c_uint32), ("max_depth", C.c_uint32)]
+
+
+class Workload(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("flags", C.c_uint32), ("task_offset", C.c_uint64),
+                ("block_threads", C.c_uint32), ("grid_ctas", C.c_uint32),
+                ("divloop", DivloopParams), ("commoncall", CommoncallParams),
+                ("mcml", MCMLParams), ("pathtrace", PathtraceParams)]
+
+
+_lib = None
+
+
+def load(path: str = LIB_PATH):
+    """Load libsr.so.  Raises FileNotFoundError if it was not built."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise FileNotFoundError(
+            f"{path} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'`"
+            " (there is no CPU fallback)")
+    L = C.CDLL(path)
+    vp, sz, u64, u32 = C.c_void_p, C.c_size_t, C.c_uint64, C.c_uint32
+    W = C.POINTER(Workload)
+    L.sr_init.argtypes = [C.c_int, vp, vp, sz]
+    L.sr_workspace_bytes.argtypes = [W, u64]; L.sr_workspace_bytes.restype = sz
+    L.sr_workspace_region.argtypes = [W, u64, C.c_int, C.POINTER(sz), C.POINTER(sz)]
+    L.sr_run.argtypes = [W, u64, u32, u64, C.c_int, u32]
+    L.sr_tally.argtypes = [C.c_int, vp, sz, C.POINTER(sz)]
+    L.sr_finalize.argtypes = []
+    L.sr_last_error.restype = C.c_char_p
+    L.sr_build_info.restype = C.c_char_p
+    fp, up = C.POINTER(C.c_float), C.POINTER(C.c_uint32)
+    L.sr_scene_build.argtypes = [fp, up, u32, fp, u32, fp, vp, sz, C.POINTER(sz)]
+    for name in ("sr_init", "sr_workspace_region", "sr_run", "sr_tally", "sr_finalize",
+                 "sr_scene_build"):
+        getattr(L, name).restype = C.c_int
+    _lib = L
+    return L
+
+
+def _check(rc: int) -> int:
+    if rc < 0:
+        raise SRError(rc, load().sr_last_error().decode())
+    return rc
+
+
+# ------------------------------------------------------------------ the C ABI, 1:1
+def sr_init(device: int, stream: int | None, workspace_ptr: int, workspace_bytes: int) -> None:
+    _check(load().sr_init(device, stream, workspace_ptr, workspace_bytes))
+
+
+def sr_workspace_bytes(w: Workload, n_threads: int) -> int:
+    return load().sr_workspace_bytes(C.byref(w), n_threads)
+
+
+def sr_workspace_region(w: Workload, n_threads: int, what: int) -> tuple[int, int]:
+    off, nb = C.c_size_t(), C.c_size_t()
+    _check(load().sr_workspace_region(C.byref(w), n_threads, what, C.byref(off), C.byref(nb)))
+    return off.value, nb.value
+
+
+def sr_run(w: Workload, n_threads: int, iters: int, seed: int, mode: int, threshold: int) -> None:
+    _check(load().sr_run(C.byref(w), n_threads, iters, seed & 0xFFFFFFFFFFFFFFFF, mode, threshold))
+
+
+def sr_tally(what: int, dst_ptr: int, dst_bytes: int) -> int:
+    written = C.c_size_t()
+    _check(load().sr_tally(what, dst_ptr, dst_bytes, C.byref(written)))
+    return written.value
+
+
+def sr_finalize() -> None:
+    _check(load().sr_finalize())
+
+
+def sr_last_error() -> str:
+    return load().sr_last_error().decode()
+
+
+def sr_build_info() -> str:
+    return load().sr_build_info().decode()
+
+
+def sr_scene_build(tris, mat, mats, cam, dst_ptr: int | None, dst_bytes: int) -> int:
+    """numpy float32 tris[n,9], uint32 mat[n], float32 mats[m,8], float32 cam[12]."""
+    import numpy as np
+    tris = np.ascontiguousarray(tris, np.float32); mat = np.ascontiguousarray(mat, np.uint32)
+    mats = np.ascontiguousarray(mats, np.float32); cam = np.ascontiguousarray(cam, np.float32)
+    fp, up = C.POINTER(C.c_float), C.POINTER(C.c_uint32)
+    needed = C.c_size_t()
+    _check(load().sr_scene_build(tris.ctypes.data_as(fp), mat.ctypes.data_as(up), len(mat),
+                                 mats.ctypes.data_as(fp), len(mats), cam.ctypes.data_as(fp),
+                                 dst_ptr, dst_bytes, C.byref(needed)))
+    return needed.value
+
+
+# ------------------------------------------------------------------ workload builders
+def divloop_workload(p_u32=1 << 29, fma_count=1000, task_offset=0, flags=0, block=0) -> Workload:
+    w = Workload(kind=WL_DIVLOOP, flags=flags, task_offset=task_offset, block_threads=block)
+    w.divloop = DivloopParams(p_u32, fma_count)
+    return w
+
+
+def commoncall_workload(fma_count=2000, split_u32=1 << 31, task_offset=0, flags=0,
+                        block=0) -> Workload:
+    w = Workload(kind=WL_COMMONCALL, flags=flags, task_offset=task_offset, block_threads=block)
+    w.commoncall = CommoncallParams(fma_count, split_u32)
+    return w
+
+
+def mcml_workload(layers, n_above=1.0, n_below=1.0, dr=0.01, dz=0.002, nr=256, nz=255,
+                  step_cap=100000, task_offset=0, flags=0, block=0, grid=0) -> Workload:
+    w = Workload(kind=WL_MCML, flags=flags, task_offset=task_offset, block_threads=block,
+                 grid_ctas=grid)
+    m = MCMLParams()
+    m.n_layers = len(layers)
+    for i, (n_, mua, mus, g, d) in enumerate(layers):
+        m.layers[i] = Layer(n_, mua, mus, g, d)
+    m.n_above, m.n_below, m.dr, m.dz = n_above, n_below, dr, dz
+    m.nr, m.nz, m.step_cap = nr, nz, step_cap
+    w.mcml = m
+    return w
+
+
+@dataclass
+class Context:
+    """A torch-owned workspace bound to libsr on the current CUDA stream."""
+    device: int
+    workspace: object   # torch.uint8 CUDA tensor
+    stream: object
+
+    @classmethod
+    def create(cls, device: int, nbytes: int, stream=None):
+        import torch
+        torch.cuda.set_device(device)
+        ws = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=f"cuda:{device}")
+        st = stream if stream is not None else torch.cuda.current_stream(device)
+        sr_init(device, st.cuda_stream, ws.data_ptr(), ws.numel())
+        return cls(device, ws, st)
+
+    def ensure(self, nbytes: int):
+        if self.workspace.numel() < nbytes:
+            import torch
+            self.workspace = torch.empty(nbytes, dtype=torch.uint8, device=f"cuda:{self.device}")
+            sr_init(self.device, self.stream.cuda_stream, self.workspace.data_ptr(), nbytes)
+
+    def region(self, w: Workload, n_threads: int, what: int, dtype):
+        """A zero-copy torch view of one workspace region of the last layout."""
+        off, nb = sr_workspace_region(w, n_threads, what)
+        return self.workspace[off:off + nb].view(dtype)

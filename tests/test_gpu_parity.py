@@ -1,0 +1,238 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle (B200 only).
+
+Bar (BASELINE.json north_star): per-thread FP outputs bit-exact (the library
+is built with --fmad=false, explicit FMAs are IEEE on both sides), integer
+tallies bit-exact, schedule counters equal to the warp simulator's.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_cgo_damanijskymg20_b200 import inputs as I
+from paper_conf_cgo_damanijskymg20_b200 import sr
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+SEEDS = I.SEEDS
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import __graft_entry__
+    __graft_entry__.build()
+    c = sr.Context.create(0, 1 << 26)
+    yield c
+    torch.cuda.synchronize()
+    sr.sr_finalize()
+
+
+def u64(t):
+    return t.cpu().numpy().view(np.uint64)
+
+
+def run_divloop(ctx, w, n, iters, seed, mode, T):
+    ctx.ensure(sr.sr_workspace_bytes(w, n))
+    sr.sr_run(w, n, iters, seed, mode, T)
+    out = ctx.region(w, n, sr.T_PERTHREAD, torch.int32).view(-1, 2).cpu().numpy()
+    cnt = u64(ctx.region(w, n, sr.T_COUNTERS, torch.int64))
+    return out[:, 0].view(np.float32).copy(), out[:, 1].view(np.uint32).copy(), cnt
+
+
+# ------------------------------------------------------------------ config 1
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 4),
+                                    (sr.SPEC_LOOP, 16), (sr.SPEC_LOOP, 32)])
+@pytest.mark.parametrize("block", [32, 64, 256])
+def test_divloop_bit_exact_small(ctx, seed, mode, T, block):
+    n, iters = 1000, 64   # 31.25 warps: several CTAs and a ragged tail
+    acc_o, cnt_o = oracle.divloop(0, n, iters, seed)
+    acc, cnt, tot = run_divloop(ctx, sr.divloop_workload(block=block), n, iters, seed, mode, T)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(cnt, cnt_o)
+    assert tot[0] == cnt_o.sum()
+
+
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 16)])
+def test_divloop_bit_exact_full_config(ctx, mode, T):
+    c = I.C1
+    acc_o, cnt_o = oracle.divloop(0, c.n_threads, c.iters, I.PRIMARY_SEED, c.p_u32, c.fma_count)
+    acc, cnt, tot = run_divloop(ctx, sr.divloop_workload(c.p_u32, c.fma_count), c.n_threads,
+                                c.iters, I.PRIMARY_SEED, mode, T)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(cnt, cnt_o)
+
+
+@pytest.mark.parametrize("kw,n,iters,off", [
+    (dict(fma_count=0), 100, 8, 0),                # no FMA: add tree only (runtime path)
+    (dict(fma_count=8), 65, 8, 0),                 # one round, runtime loop
+    (dict(fma_count=2000), 33, 16, 0),             # other compile-time instantiation
+    (dict(p_u32=0), 64, 16, 0),                    # never wants
+    (dict(p_u32=0xFFFFFFFF), 64, 16, 0),           # always wants
+    (dict(), 1, 64, 0),                            # a single thread
+    (dict(), 100, 0, 0),                           # zero iterations
+    (dict(), 100, 16, (1 << 40) + 12345),          # 64-bit task ids
+])
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 16), (sr.SPEC_LOOP, 32)])
+def test_divloop_edge_cases(ctx, kw, n, iters, off, mode, T):
+    w = sr.divloop_workload(task_offset=off, **kw)
+    p = dict(p_u32=1 << 29, fma_count=1000); p.update(kw)
+    acc_o, cnt_o = oracle.divloop(off, n, iters, 7, p["p_u32"], p["fma_count"])
+    acc, cnt, _ = run_divloop(ctx, w, n, iters, 7, mode, T)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(cnt, cnt_o)
+
+
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 16),
+                                    (sr.SPEC_LOOP, 32)])
+def test_divloop_schedule_matches_simulator(ctx, mode, T):
+    """Per-warp rounds / releases / lane counts equal oracle part 2 exactly."""
+    n, iters = 2000, 64
+    w = sr.divloop_workload(flags=sr.F_SCHED, block=64)
+    run_divloop(ctx, w, n, iters, I.PRIMARY_SEED, mode, T)
+    sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    want = oracle.divloop_wants(0, n, iters, I.PRIMARY_SEED)
+    for wi in range((n + 31) // 32):
+        ww = want[32 * wi:32 * wi + 32]
+        s = oracle.ws_divloop(ww, oracle.PDOM if mode == sr.PDOM else oracle.SPEC_LOOP, T)
+        g = sched[wi]
+        assert (g[1], g[2]) == s["EXPENSIVE"], wi
+        if mode == sr.SPEC_LOOP:
+            assert g[0] == s["rounds"], wi
+            assert (g[3], g[4]) == s["ADVANCE"] and s["PROLOG"] == s["ADVANCE"], wi
+
+
+# ------------------------------------------------------------------ config 2
+def run_cc(ctx, w, n, iters, seed, mode):
+    ctx.ensure(sr.sr_workspace_bytes(w, n))
+    sr.sr_run(w, n, iters, seed, mode, 0)
+    y = ctx.region(w, n, sr.T_PERTHREAD, torch.float32).cpu().numpy().copy()
+    return y, u64(ctx.region(w, n, sr.T_COUNTERS, torch.int64))
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("mode", [sr.PDOM, sr.SPEC_CALL])
+@pytest.mark.parametrize("n,iters,block", [(1000, 1, 256), (77, 3, 32), (4096, 1, 1024)])
+def test_commoncall_bit_exact(ctx, seed, mode, n, iters, block):
+    y_o, arm = oracle.commoncall(0, n, iters, seed)
+    y, cnt = run_cc(ctx, sr.commoncall_workload(block=block), n, iters, seed, mode)
+    assert np.array_equal(y.view(np.uint32), y_o.view(np.uint32))
+    if iters == 1:
+        assert cnt[0] == arm.sum()
+
+
+@pytest.mark.parametrize("mode", [sr.PDOM, sr.SPEC_CALL])
+def test_commoncall_bit_exact_full_config(ctx, mode):
+    c = I.C2
+    y_o, _ = oracle.commoncall(0, c.n_threads, c.iters, I.PRIMARY_SEED, c.split_u32, c.fma_count)
+    y, _ = run_cc(ctx, sr.commoncall_workload(c.fma_count, c.split_u32), c.n_threads, c.iters,
+                  I.PRIMARY_SEED, mode)
+    assert np.array_equal(y.view(np.uint32), y_o.view(np.uint32))
+
+
+@pytest.mark.parametrize("mode", [sr.PDOM, sr.SPEC_CALL])
+def test_commoncall_schedule_matches_simulator(ctx, mode):
+    n = 1000
+    w = sr.commoncall_workload(flags=sr.F_SCHED)
+    run_cc(ctx, w, n, 1, I.PRIMARY_SEED, mode)
+    sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    _, arm = oracle.commoncall(0, n, 1, I.PRIMARY_SEED)
+    for wi in range((n + 31) // 32):
+        s = oracle.ws_commoncall(arm[32 * wi:32 * wi + 32],
+                                 oracle.PDOM if mode == sr.PDOM else oracle.SPEC_CALL)
+        assert (sched[wi][1], sched[wi][2]) == s["CALL"], wi
+
+
+# ------------------------------------------------------------------ configs 3/5
+def mc_oracle(m, id0, count, seed):
+    p = oracle.mc_params(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap)
+    return oracle.mcml(p, id0, count, seed, steps=True)
+
+
+def mc_workload(m, **kw):
+    return sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap, **kw)
+
+
+def run_mc(ctx, w, n, iters, seed, mode, T, m):
+    ctx.ensure(sr.sr_workspace_bytes(w, n))
+    sr.sr_run(w, n, iters, seed, mode, T)
+    g = u64(ctx.region(w, n, sr.T_GRID, torch.int64))
+    nA = m.nz * m.nr
+    cnt = u64(ctx.region(w, n, sr.T_COUNTERS, torch.int64))
+    return dict(A=g[:nA], Rd=g[nA:nA + m.nr], Tt=g[nA + m.nr:], counters=cnt[:8])
+
+
+def assert_mc_equal(got, ref):
+    assert np.array_equal(got["A"], ref["A"].ravel())
+    assert np.array_equal(got["Rd"], ref["Rd"])
+    assert np.array_equal(got["Tt"], ref["Tt"])
+    assert np.array_equal(got["counters"], ref["counters_raw"])
+
+
+@pytest.mark.parametrize("seed", SEEDS)
+@pytest.mark.parametrize("flags", [0, sr.F_STATIC])
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 8),
+                                    (sr.SPEC_LOOP, 32)])
+def test_mcml_bit_exact_small(ctx, seed, flags, mode, T):
+    m = I.C3
+    nt, it = 300, 5   # ragged: 9.4 warps, 1500 photons
+    ref = mc_oracle(m, 0, nt * it, seed)
+    got = run_mc(ctx, mc_workload(m, flags=flags, block=128), nt, it, seed, mode, T, m)
+    assert_mc_equal(got, ref)
+
+
+@pytest.mark.parametrize("name", ["BEER_LAMBERT", "NO_ABSORPTION", "VAN_DE_HULST"])
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 32)])
+def test_mcml_bit_exact_pin_workloads(ctx, name, mode, T):
+    m = getattr(I, name)
+    ref = mc_oracle(m, 5000, 4096, 11)
+    got = run_mc(ctx, mc_workload(m, task_offset=5000), 512, 8, 11, mode, T, m)
+    assert_mc_equal(got, ref)
+
+
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 4), (sr.SPEC_LOOP, 32)])
+def test_mcml_schedule_matches_simulator(ctx, mode, T):
+    m = I.C3
+    nt, it = 96, 6
+    w = mc_workload(m, flags=sr.F_STATIC | sr.F_SCHED, block=32)
+    run_mc(ctx, w, nt, it, 3, mode, T, m)
+    sched = ctx.region(w, nt, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    ref = mc_oracle(m, 0, nt * it, 3)
+    steps = ref["steps"].reshape(it, nt).T     # photon l + k*nt -> [lane, k]
+    for wi in range(nt // 32):
+        ns = steps[32 * wi:32 * wi + 32]
+        s = oracle.ws_loopmerge(ns, oracle.PDOM if mode == sr.PDOM else oracle.SPEC_LOOP, T)
+        g = sched[wi]
+        assert (g[1], g[2]) == s["STEP"], wi
+        if mode == sr.SPEC_LOOP:
+            assert g[0] == s["rounds"] and (g[3], g[4]) == s["LAUNCH"], wi
+
+
+def test_mcml_full_size_invariants(ctx):
+    """Config 3 at full size in the bench launch configuration: PDOM == SPEC
+    (T=32, 16) bit for bit, == the sum of two shards, and a slice far into the
+    id range equals the oracle."""
+    m = I.C3
+    nt, it = m.n_threads, m.iters
+    w = mc_workload(m)
+    full = run_mc(ctx, w, nt, it, I.PRIMARY_SEED, sr.SPEC_LOOP, 32, m)
+    assert full["counters"][0] == nt * it
+    for mode, T in ((sr.PDOM, 0), (sr.SPEC_LOOP, 16)):
+        o = run_mc(ctx, w, nt, it, I.PRIMARY_SEED, mode, T, m)
+        for k in full:
+            assert np.array_equal(o[k], full[k]), (mode, T, k)
+    half = nt // 2
+    a = run_mc(ctx, mc_workload(m), half, it, I.PRIMARY_SEED, sr.SPEC_LOOP, 32, m)
+    b = run_mc(ctx, mc_workload(m, task_offset=half * it), nt - half, it, I.PRIMARY_SEED,
+               sr.SPEC_LOOP, 32, m)
+    for k in full:
+        assert np.array_equal(a[k] + b[k], full[k]), k
+    c = full["counters"]
+    assert c[2] + c[3] + c[4] + c[6] + c[7] == nt * it   # every photon ends exactly once
+    off = 9_000_000
+    ref = mc_oracle(m, off, 20000, I.PRIMARY_SEED)
+    got = run_mc(ctx, mc_workload(m, task_offset=off), 20000, 1, I.PRIMARY_SEED, sr.SPEC_LOOP,
+                 32, m)
+    assert_mc_equal(got, ref)
