@@ -1,0 +1,404 @@
+#!/usr/bin/env python
+"""Benchmark of the Speculative Reconvergence hot path on B200.
+
+Contract (driver): ``python bench.py --gpus N --steps K --warmup W`` prints ONE
+JSON line on rank 0.  For N > 1 it is launched under torch.distributed.run, one
+process per GPU, NCCL.
+
+Headline workload: Monte Carlo photon transport in the
+3-layer slab (BASELINE.json configs[2]: 10^7 photons per GPU), Loop Merge
+(SR_SPEC_LOOP, T=32) -- one step = one sr_run over the rank's photon shard plus,
+for N > 1, one NCCL all-reduce of the integer tallies (configs[4] is this run
+weak-scaled: N x 10^7 photons).  The PDOM kernel is timed the same way
+("pdom" key).  At N = 1 the two microbenchmarks (configs[0], configs[1]) are
+timed too ("configs" key), PDOM vs SPEC.
+
+``--impl reference`` times the CPU oracle (oracle/, plain single-threaded C) on
+a bounded sample of the same workload instead -- the reference arm of this
+tier (there is no reference program to install).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "samples/sec and ncu SIMT efficiency, speculative vs PDOM, at 1/2/4/8 B200"
+UNIT = "photons/s"
+PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
+PROFILE_CONST = os.path.join(ROOT, "profiles", "work_per_unit.json")
+L2_FLUSH_BYTES = 256 << 20  # > 126 MB L2
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--threshold", type=int, default=32)
+    ap.add_argument("--photons-per-gpu", type=int, default=0,
+                    help="override the per-rank photon count (default: configs[2] = 10^7)")
+    ap.add_argument("--no-configs", action="store_true", help="skip the microbenchmark lines")
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    return ap.parse_args()
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+# ---------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi sampling DURING the timed region (B200_PROFILING.md)."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+            self.t.join(timeout=2)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[1]) for r in self.rows if len(r) > 1 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) > 2 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for i, n in enumerate(names):
+                if len(r) > 5 + i and r[5 + i].lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "samples": len(self.rows)}
+
+
+# ---------------------------------------------------------------- timing
+class Timer:
+    """Per-step CUDA events on the launching stream; an L2 flush (a 256 MB
+    write) between timed steps, outside the events."""
+
+    def __init__(self, torch, stream):
+        self.torch = torch
+        self.stream = stream
+        self.flush_buf = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device=stream.device)
+
+    def flush(self):
+        with self.torch.cuda.stream(self.stream):
+            self.flush_buf.fill_(1)
+
+    def time_steps(self, fn, steps, warmup, barrier=None):
+        torch = self.torch
+        for _ in range(warmup):
+            self.flush()
+            fn()
+        torch.cuda.synchronize()
+        if barrier:
+            barrier()
+        torch.cuda.synchronize()
+        ms = []
+        for _ in range(steps):
+            self.flush()
+            s = torch.cuda.Event(enable_timing=True)
+            e = torch.cuda.Event(enable_timing=True)
+            s.record(self.stream)
+            fn()
+            e.record(self.stream)
+            e.synchronize()
+            ms.append(s.elapsed_time(e))
+        torch.cuda.synchronize()
+        if barrier:
+            barrier()
+        torch.cuda.synchronize()
+        return ms
+
+
+def load_json(path):
+    try:
+        with open(path) as f:
+            return json.load(f)
+    except (OSError, ValueError):
+        return None
+
+
+# ---------------------------------------------------------------- reference arm
+def cpu_sample(photons: int, seed: int):
+    """The oracle, as it stands, single-threaded on this host: photons/s."""
+    import oracle
+    from paper_conf_cgo_damanijskymg20_b200 import inputs as I
+    m = I.C3
+    p = oracle.mc_params(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap)
+    t = time.perf_counter()
+    oracle.mcml(p, 0, photons, seed)
+    return photons / (time.perf_counter() - t)
+
+
+def run_reference(args):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return
+    from paper_conf_cgo_damanijskymg20_b200 import inputs as I
+    sample = 16384  # ~0.6 s of oracle work per step
+    for _ in range(args.warmup):
+        cpu_sample(sample // 8, I.PRIMARY_SEED)
+    vals = [cpu_sample(sample, I.PRIMARY_SEED) for _ in range(args.steps)]
+    v = statistics.median(vals)
+    out = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": sample / v * 1e3,
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+           "data": "synthetic",
+           "config": {"workload": "mcml-3layer (configs[2]) photon ids [0,16384) per step",
+                      "photons_per_gpu": I.C3.n_photons, "seed": I.PRIMARY_SEED},
+           "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                            "sample": f"{sample} photons of configs[2] per step, single thread"},
+           "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+# ---------------------------------------------------------------- our arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_cgo_damanijskymg20_b200 import inputs as I
+    from paper_conf_cgo_damanijskymg20_b200 import sr
+
+    ws_n, rank, local = dist_env()
+    if ws_n > 1:
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    torch.cuda.set_device(local)
+    dev = torch.device(f"cuda:{local}")
+    stream = torch.cuda.Stream(device=dev)
+    sr.load()  # raises if libsr.so is missing: no fallback
+
+    m = I.C3
+    per_rank = args.photons_per_gpu or m.n_photons
+    iters = m.iters
+    nt = (per_rank + iters - 1) // iters
+    per_rank = nt * iters
+    T = args.threshold
+    w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
+                         task_offset=rank * per_rank)
+    nbytes = sr.sr_workspace_bytes(w, nt)
+    ctx = sr.Context.create(local, nbytes, stream)
+    off, tb = sr.sr_workspace_region(w, nt, sr.T_GRID)
+    _, cb = sr.sr_workspace_region(w, nt, sr.T_COUNTERS)
+    tallies = ctx.workspace[off:off + tb + cb].view(torch.int64)  # GRID + COUNTERS, contiguous
+    barrier = (lambda: dist.barrier()) if ws_n > 1 else None
+    timer = Timer(torch, stream)
+
+    def step(mode, thr):
+        sr.sr_run(w, nt, iters, I.PRIMARY_SEED, mode, thr)
+        if ws_n > 1:
+            with torch.cuda.stream(stream):
+                dist.all_reduce(tallies, op=dist.ReduceOp.SUM)
+
+    # device-timed region, SPEC (headline) with clocks sampled during it
+    with ClockSampler(local) as clk:
+        ms_spec = timer.time_steps(lambda: step(sr.SPEC_LOOP, T), args.steps, args.warmup, barrier)
+    ms_pdom = timer.time_steps(lambda: step(sr.PDOM, 0), args.steps, args.warmup, barrier)
+
+    def max_over_ranks(x):
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        if ws_n > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    t_spec = max_over_ranks(statistics.mean(ms_spec))
+    t_pdom = max_over_ranks(statistics.mean(ms_pdom))
+    total = per_rank * ws_n
+    value = total / (t_spec * 1e-3)
+    pdom_value = total / (t_pdom * 1e-3)
+
+    # end to end through the public API: sr_run + (all-reduce) + sr_tally into
+    # pinned host memory, host wall clock per step, max over ranks
+    host = torch.empty(tb + cb, dtype=torch.uint8, pin_memory=True)
+    h2d = 0
+    import ctypes
+    h2d = ctypes.sizeof(sr.Workload)   # the step's inputs: the workload descriptor
+    e2e_ms = []
+    for i in range(args.warmup + args.steps):
+        torch.cuda.synchronize()
+        if barrier:
+            barrier()
+        t0 = time.perf_counter()
+        step(sr.SPEC_LOOP, T)
+        sr.sr_tally(sr.T_GRID, host.data_ptr(), tb)
+        sr.sr_tally(sr.T_COUNTERS, host.data_ptr() + tb, cb)
+        t1 = time.perf_counter()
+        if i >= args.warmup:
+            e2e_ms.append((t1 - t0) * 1e3)
+    t_e2e = max_over_ranks(statistics.mean(e2e_ms))
+    counters = host[tb:tb + cb].view(torch.int64).numpy()
+    steps_total = int(counters[1])  # after all-reduce: whole job
+    assert int(counters[0]) == total, "photon count mismatch"
+
+    # schedule-level efficiency of the common code (instrumented kernels, outside timing)
+    def region_eff(mode, thr):
+        wi = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz,
+                              m.step_cap, task_offset=rank * per_rank, flags=sr.F_SCHED)
+        ctx.ensure(sr.sr_workspace_bytes(wi, nt))
+        ni = min(nt, 32768)
+        sr.sr_run(wi, ni, iters, I.PRIMARY_SEED, mode, thr)
+        s = ctx.region(wi, ni, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS)
+        s = s.cpu().numpy().astype("int64")
+        rel, lanes = s[:, 1].sum(), s[:, 2].sum()
+        return float(lanes / (32.0 * rel)) if rel else None
+
+    eff_spec = region_eff(sr.SPEC_LOOP, T)
+    eff_pdom = region_eff(sr.PDOM, 0)
+
+    peaks = load_json(PEAKS_FILE) or {}
+    consts = load_json(PROFILE_CONST) or {}
+    clocks = clk.summary()
+    result = None
+    if rank == 0:
+        # roofline: issue-bound (plain ALU), algorithmic thread-instructions =
+        # PDOM thread-instructions per photon-step (ncu, profiles/) x steps
+        ipu = consts.get("mcml_thread_inst_per_step")
+        f_mhz = peaks.get("sm_max_mhz", 1965.0)
+        peak = 32 * 4 * 148 * f_mhz * 1e6 / 1e12   # T thread-inst/s
+        rl = None
+        if ipu:
+            ach = ipu * steps_total / ws_n / (t_spec * 1e-3) / 1e12
+            rl = {"bound": "alu", "achieved": ach, "peak": peak, "unit": "Tthread-inst/s",
+                  "frac": ach / peak, "traffic": consts.get("mcml_spec_dram_bytes_per_launch"),
+                  "kernel": "mcml_spec",
+                  "peak_basis": f"592 SMSPs x 32 lanes x {f_mhz:.0f} MHz (sm_max_mhz of measured)",
+                  "work_basis": "profiles/work_per_unit.json: PDOM thread-inst per photon step (ncu)"}
+        result = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws_n, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": t_spec, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": "mcml-3layer (configs[2] per GPU; N GPUs = configs[4] weak-scaled)",
+                       "photons_per_gpu": per_rank, "lanes": nt, "photons_per_lane": iters,
+                       "threshold": T, "mode": "SPEC_LOOP", "seed": I.PRIMARY_SEED,
+                       "l2": "flushed (256 MB write) between timed steps",
+                       "parallelism": f"dp{ws_n} (photon-id shards + 1 NCCL int64 all-reduce)"},
+            "pdom": {"value": pdom_value, "unit": UNIT, "ms_per_step": t_pdom},
+            "speedup_vs_pdom": value / pdom_value,
+            "common_region_efficiency": {"pdom": eff_pdom, "spec": eff_spec,
+                                         "source": "per-warp schedule counters (SR_F_SCHED)"},
+            "steps_per_photon": steps_total / total,
+            "clocks": clocks,
+            "e2e": {"value": total / (t_e2e * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": tb + cb},
+            "gpu_launches": args.steps,
+            "roofline": rl,
+        }
+        simt = load_json(os.path.join(ROOT, "profiles", "simt_efficiency.json"))
+        if simt:
+            result["simt_efficiency_ncu"] = simt
+    if ws_n > 1:
+        dist.barrier()
+    if rank == 0 and ws_n == 1 and not args.no_configs:
+        result["configs"] = microbench_configs(torch, sr, I, ctx, stream, timer, args)
+    if rank == 0 and ws_n == 1 and not args.no_cpu:
+        t = time.perf_counter()
+        n_cpu, v_cpu = 1024, cpu_sample(1024, I.PRIMARY_SEED)
+        n_cpu = max(1024, int(v_cpu * 15))  # ~15 s of single-core oracle work
+        v_cpu = cpu_sample(n_cpu, I.PRIMARY_SEED)
+        result["cpu_baseline"] = {"value": v_cpu, "unit": UNIT, "cores": 1, "kind": "oracle",
+                                  "sample": f"photon ids [0,{n_cpu}) of configs[2], single thread",
+                                  "seconds": time.perf_counter() - t}
+    if rank == 0:
+        print(json.dumps(result), flush=True)
+    sr.sr_finalize()
+    if ws_n > 1:
+        dist.destroy_process_group()
+
+
+def microbench_configs(torch, sr, I, ctx, stream, timer, args):
+    """configs[0] and configs[1]: PDOM vs SPEC, CUDA-graph replays of R launches."""
+    out = {}
+    peaks = load_json(PEAKS_FILE) or {}
+    f_mhz = peaks.get("sm_max_mhz", 1965.0)
+    fma_peak = 128 * 148 * f_mhz * 1e6  # FP32 FMA/s (FFMA2 = 2 per lane)
+
+    def graph_time(w, n, iters, mode, thr, reps=20):
+        ctx.ensure(sr.sr_workspace_bytes(w, n))
+        g = torch.cuda.CUDAGraph()
+        cap = torch.cuda.Stream(device=stream.device)
+        sr.sr_init(ctx.device, cap.cuda_stream, ctx.workspace.data_ptr(), ctx.workspace.numel())
+        sr.sr_run(w, n, iters, I.PRIMARY_SEED, mode, thr)  # warm (module load, attributes)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=cap):
+            for _ in range(reps):
+                sr.sr_run(w, n, iters, I.PRIMARY_SEED, mode, thr)
+        sr.sr_init(ctx.device, stream.cuda_stream, ctx.workspace.data_ptr(), ctx.workspace.numel())
+        ms = timer.time_steps(lambda: g.replay(), max(args.steps, 5), args.warmup)
+        return statistics.median(ms) / reps
+
+    c = I.C1
+    w = sr.divloop_workload(c.p_u32, c.fma_count)
+    n_units = c.n_threads * c.iters
+    exp_calls = None
+    res = {}
+    for name, mode, thr in (("pdom", sr.PDOM, 0), ("spec_t16", sr.SPEC_LOOP, 16),
+                            ("spec_t32", sr.SPEC_LOOP, 32)):
+        t = graph_time(w, c.n_threads, c.iters, mode, thr)
+        sr.sr_run(w, c.n_threads, c.iters, I.PRIMARY_SEED, mode, thr)
+        exp_calls = int(ctx.region(w, c.n_threads, sr.T_COUNTERS, torch.int64)[0].item())
+        res[name] = {"value": n_units / (t * 1e-3), "unit": "thread-iterations/s", "ms": t,
+                     "fma_frac_of_peak": exp_calls * c.fma_count / (t * 1e-3) / fma_peak}
+    res["speedup_t16_vs_pdom"] = res["spec_t16"]["value"] / res["pdom"]["value"]
+    res["expensive_calls"] = exp_calls
+    out["divloop"] = res
+
+    c = I.C2
+    w = sr.commoncall_workload(c.fma_count, c.split_u32)
+    res = {}
+    for name, mode in (("pdom", sr.PDOM), ("spec_call", sr.SPEC_CALL)):
+        t = graph_time(w, c.n_threads, c.iters, mode, 0, reps=5)
+        res[name] = {"value": c.n_threads / (t * 1e-3), "unit": "threads/s", "ms": t,
+                     "fma_frac_of_peak": c.n_threads * c.fma_count / (t * 1e-3) / fma_peak}
+    res["speedup_vs_pdom"] = res["spec_call"]["value"] / res["pdom"]["value"]
+    out["commoncall"] = res
+    return out
+
+
+if __name__ == "__main__":
+    main()
