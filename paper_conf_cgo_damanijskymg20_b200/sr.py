@@ -207,4 +207,5 @@ class Context:
     def region(self, w: Workload, n_threads: int, what: int, dtype):
         """A zero-copy torch view of one workspace region of the last layout."""
         off, nb = sr_workspace_region(w, n_threads, what)
+        self.stream.synchronize()  # the library works on self.stream, not torch's current one
         return self.workspace[off:off + nb].view(dtype)

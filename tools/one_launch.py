@@ -1,0 +1,50 @@
+"""Launch each hot-path kernel once (for ncu); no timing, no oracle.
+
+usage: python tools/one_launch.py [divloop] [commoncall] [mcml] [--photons N] [--sched]
+"""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+from paper_conf_cgo_damanijskymg20_b200 import inputs as I  # noqa: E402
+from paper_conf_cgo_damanijskymg20_b200 import sr  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("what", nargs="*", default=["divloop", "commoncall", "mcml"])
+ap.add_argument("--photons", type=int, default=I.C3.n_photons)
+ap.add_argument("--modes", default="pdom,spec")
+ap.add_argument("--threshold", type=int, default=32)
+ap.add_argument("--static", action="store_true")
+a = ap.parse_args()
+modes = a.modes.split(",")
+ctx = sr.Context.create(0, 1 << 20)
+seed = I.PRIMARY_SEED
+if "divloop" in a.what:
+    c = I.C1
+    w = sr.divloop_workload(c.p_u32, c.fma_count)
+    ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
+    for md in modes:
+        sr.sr_run(w, c.n_threads, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
+                  0 if md == "pdom" else c.threshold)
+if "commoncall" in a.what:
+    c = I.C2
+    w = sr.commoncall_workload(c.fma_count, c.split_u32)
+    ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
+    for md in modes:
+        sr.sr_run(w, c.n_threads, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_CALL, 0)
+if "mcml" in a.what:
+    m = I.C3
+    nt = a.photons // m.iters
+    w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
+                         flags=sr.F_STATIC if a.static else 0)
+    ctx.ensure(sr.sr_workspace_bytes(w, nt))
+    for md in modes:
+        sr.sr_run(w, nt, m.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
+                  0 if md == "pdom" else a.threshold)
+torch.cuda.synchronize()
+sr.sr_finalize()
+print("ok")
