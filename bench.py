@@ -239,7 +239,9 @@ def main():
     # device-timed region, SPEC (headline) with clocks sampled during it
     with ClockSampler(local) as clk:
         ms_spec = timer.time_steps(lambda: step(sr.SPEC_LOOP, T), args.steps, args.warmup, barrier)
+    launch_spec = sr.sr_last_launch()
     ms_pdom = timer.time_steps(lambda: step(sr.PDOM, 0), args.steps, args.warmup, barrier)
+    launch_pdom = sr.sr_last_launch()
 
     def max_over_ranks(x):
         t = torch.tensor([x], dtype=torch.float64, device=dev)
@@ -317,6 +319,7 @@ def main():
                        "photons_per_gpu": per_rank, "lanes": nt, "photons_per_lane": iters,
                        "threshold": T, "mode": "SPEC_LOOP", "seed": I.PRIMARY_SEED,
                        "l2": "flushed (256 MB write) between timed steps",
+                       "launch": launch_spec, "launch_pdom": launch_pdom,
                        "parallelism": f"dp{ws_n} (photon-id shards + 1 NCCL int64 all-reduce)"},
             "pdom": {"value": pdom_value, "unit": UNIT, "ms_per_step": t_pdom},
             "speedup_vs_pdom": value / pdom_value,

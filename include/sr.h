@@ -162,6 +162,25 @@ SR_API const char* sr_last_error(void);
 /* Library build identification: "sm_100a <nvcc version> <flags>". */
 SR_API const char* sr_build_info(void);
 
+/* Launch configuration of the last kernel sr_run enqueued:
+ * out[0] = CTAs, out[1] = threads per CTA, out[2] = dynamic shared memory
+ * bytes per CTA, out[3] = kernels launched by that sr_run.
+ * SR_E_STATE if no run happened since sr_init. */
+SR_API int sr_last_launch(uint32_t out[4]);
+
+/* Diagnostics: evaluate one device building block of the hot path element
+ * by element, out[i] = fn(x[i]), on the context stream (no synchronize).
+ * x_dev, out_dev: device arrays of n floats, caller-owned.
+ *   SR_FN_LOGF            sr_logf(x), x in (0,1]            (R5)
+ *   SR_FN_SIN2PI/COS2PI   sin/cos(2 pi x), x = k 2^-24       (R5)
+ *   SR_FN_EXPENSIVE_1000  Expensive() of config 1 started at x (R3)
+ *   SR_FN_EXPENSIVE_2000  foo() of config 2 started at x     (R4)
+ * Errors: SR_E_STATE before sr_init; SR_E_INVALID (unknown fn, NULL with
+ * n > 0); SR_E_CUDA. */
+enum { SR_FN_LOGF = 0, SR_FN_SIN2PI = 1, SR_FN_COS2PI = 2, SR_FN_EXPENSIVE_1000 = 3,
+       SR_FN_EXPENSIVE_2000 = 4 };
+SR_API int sr_math_eval(int fn, const float* x_dev, float* out_dev, uint64_t n);
+
 /* PATHTRACE scene (config 4): build the BVH over a caller-provided triangle
  * soup on the host and write the device scene image.
  *   tris       host, n_tris x 9 floats (v0, v1, v2 xyz), caller-owned

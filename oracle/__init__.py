@@ -116,6 +116,15 @@ def philox(ctr, key):
     return out
 
 
+def eval_batch(fn: int, x):
+    x = np.ascontiguousarray(x, np.float32)
+    out = np.empty_like(x)
+    L = lib()
+    L.or_eval_batch.argtypes = [C.c_int, C.POINTER(C.c_float), C.POINTER(C.c_float), C.c_uint64]
+    L.or_eval_batch(fn, _p(x, C.c_float), _p(out, C.c_float), x.size)
+    return out
+
+
 def sr_logf(x: float) -> float:
     return lib().or_sr_logf(x)
 

@@ -47,6 +47,9 @@ void  or_sr_sincos2pif(float xi, float* s, float* c);  /* xi = k*2^-24, k<2^24  
  * returns max |error| in units of the float ulp of the exact result. */
 double or_sweep_logf_ulp(void);
 double or_sweep_sincos2pif_ulp(void);
+/* out[i] = fn(x[i]); fn: 0 log, 1 sin2pi, 2 cos2pi, 3 Expensive(1000 FMAs),
+ * 4 Expensive(2000 FMAs) */
+void or_eval_batch(int fn, const float* x, float* out, uint64_t n);
 
 /* ---- divloop.c : config 1, divergent condition in a loop (Fig. 2(a)). */
 typedef struct { uint32_t p_u32, fma_count; } or_divloop_params;

@@ -34,12 +34,12 @@ def nvcc_version() -> str:
     return out.strip().splitlines()[-1].split(",")[0].replace("Build ", "") if out else "?"
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, defines=(), lib: str = LIB) -> str:
     srcs = sources()
     newest = max(os.path.getmtime(p) for p in srcs + headers() + [__file__])
-    if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= newest:
-        return LIB
-    objdir = os.path.join(HERE, "build")
+    if not force and os.path.exists(lib) and os.path.getmtime(lib) >= newest:
+        return lib
+    objdir = os.path.join(HERE, "build", os.path.basename(lib))
     os.makedirs(objdir, exist_ok=True)
     ver = nvcc_version()
     objs = []
@@ -47,7 +47,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     for s in srcs:
         o = os.path.join(objdir, os.path.basename(s) + ".o")
         objs.append(o)
-        cmd = [NVCC, *ARCH, *FLAGS, f'-DSR_NVCC_VERSION="{ver}"', "-I", os.path.join(ROOT, "include"),
+        cmd = [NVCC, *ARCH, *FLAGS, f'-DSR_NVCC_VERSION="{ver}"', "-I", os.path.join(ROOT, "include"), *[f"-D{d}" for d in defines],
                "-dc" if False else "-c", s, "-o", o]
         if verbose:
             cmd += ["-Xptxas", "-v"]
@@ -59,13 +59,13 @@ def build(force: bool = False, verbose: bool = False) -> str:
         logs.append(out)
         if p.returncode != 0:
             raise RuntimeError(f"nvcc failed on {s}:\n{out}")
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = lib + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs,
                            "-Xlinker", "--exclude-libs,ALL"])
-    os.replace(tmp, LIB)
+    os.replace(tmp, lib)
     if verbose:
         print("".join(logs))
-    return LIB
+    return lib
 
 
 if __name__ == "__main__":

@@ -125,6 +125,7 @@ cudaError_t launch_t(const LaunchCtx& c, const CallArgs& a, int mode) {
   const uint64_t grid = (a.n + block - 1) / block;
   if (grid > 0x7fffffffull) return cudaErrorInvalidConfiguration;
   const bool spec = mode == SR_SPEC_CALL;
+  record_launch((uint32_t)grid, block, 0);
 #define SR_CC(R)                                                                        \
   (spec ? commoncall_spec<R, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a)        \
         : commoncall_pdom<R, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a))

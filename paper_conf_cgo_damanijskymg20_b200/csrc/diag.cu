@@ -1,0 +1,41 @@
+// diag.cu -- sr_math_eval: evaluate one device building block of the hot path
+// element-wise, so tests can compare the GPU's sr_logf / sr_sincos2pif /
+// Expensive() with the CPU oracle bit for bit over every input the RNG can
+// produce (readings R3, R5).
+#include "sr_device.cuh"
+#include "sr_internal.h"
+
+namespace sr {
+namespace {
+
+__global__ void math_eval_kernel(int fn, const float* __restrict__ x, float* __restrict__ out,
+                                 uint64_t n) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    const float v = x[i];
+    float r;
+    switch (fn) {
+      case SR_FN_LOGF: r = sr_logf(v); break;
+      case SR_FN_SIN2PI: { float s, c; sr_sincos2pif(v, s, c); r = s; break; }
+      case SR_FN_COS2PI: { float s, c; sr_sincos2pif(v, s, c); r = c; break; }
+      case SR_FN_EXPENSIVE_1000: r = expensive<125>(v, 125); break;
+      case SR_FN_EXPENSIVE_2000: r = expensive<250>(v, 250); break;
+      default: r = 0.0f; break;
+    }
+    out[i] = r;
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_math_eval(cudaStream_t st, int sm_count, int fn, const float* x, float* out,
+                             uint64_t n) {
+  const uint64_t want = (n + 255) / 256;
+  const uint64_t cap = (uint64_t)sm_count * 16;
+  const unsigned grid = (unsigned)(want < cap ? (want ? want : 1) : cap);
+  record_launch(grid, 256, 0);
+  math_eval_kernel<<<grid, 256, 0, st>>>(fn, x, out, n);
+  return cudaGetLastError();
+}
+
+}  // namespace sr

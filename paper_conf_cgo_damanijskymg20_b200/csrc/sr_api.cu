@@ -29,6 +29,7 @@ struct Context {
 };
 Context g_ctx;
 std::mutex g_mu;
+uint32_t g_launch[4];  // grid, block, smem, kernels of the current/last sr_run
 
 int fail(int code, const std::string& msg) {
   g_err = msg;
@@ -77,6 +78,13 @@ uint32_t default_block(const sr_workload& w) {
 }
 
 }  // namespace
+
+void record_launch(uint32_t grid, uint32_t block, uint32_t smem_bytes) {
+  g_launch[0] = grid;
+  g_launch[1] = block;
+  g_launch[2] = smem_bytes;
+  g_launch[3] += 1;
+}
 
 Layout layout_of(const sr_workload& w, uint64_t n) {
   Layout L{};
@@ -129,6 +137,27 @@ const char* sr_build_info(void) {
 #define SR_NVCC_VERSION "unknown"
 #endif
   return "libsr sm_100a nvcc " SR_NVCC_VERSION " --fmad=false -O3 -lineinfo";
+}
+
+int sr_math_eval(int fn, const float* x_dev, float* out_dev, uint64_t n) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  g_err.clear();
+  if (fn < SR_FN_LOGF || fn > SR_FN_EXPENSIVE_2000) return fail(SR_E_INVALID, "unknown fn");
+  if (n && (!x_dev || !out_dev)) return fail(SR_E_INVALID, "NULL array");
+  if (!g_ctx.live) return fail(SR_E_STATE, "sr_math_eval before sr_init");
+  if (!n) return SR_OK;
+  const cudaError_t e = launch_math_eval(g_ctx.stream, g_ctx.sm_count, fn, x_dev, out_dev, n);
+  if (e != cudaSuccess) return fail_cuda(e, "sr_math_eval");
+  return SR_OK;
+}
+
+int sr_last_launch(uint32_t out[4]) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  g_err.clear();
+  if (!out) return fail(SR_E_INVALID, "out is NULL");
+  if (!g_ctx.have_run) return fail(SR_E_STATE, "no sr_run since sr_init");
+  for (int i = 0; i < 4; ++i) out[i] = g_launch[i];
+  return SR_OK;
 }
 
 int sr_init(int device, void* cuda_stream, void* workspace_dev, size_t workspace_bytes) {
@@ -200,6 +229,7 @@ int sr_run(const sr_workload* w, uint64_t n_threads, uint32_t iters, uint64_t se
                                 std::to_string(L.total));
   LaunchCtx c{g_ctx.stream, g_ctx.ws, L, g_ctx.sm_count, default_block(*w)};
   cudaError_t e;
+  g_launch[3] = 0;
   // zero the outputs of this run (per-thread outputs are fully overwritten)
   for (int r : {SR_T_GRID, SR_T_COUNTERS, SR_T_SCHED, SR_T_SCRATCH}) {
     if (!L.bytes[r]) continue;

@@ -29,6 +29,9 @@ struct LaunchCtx {
   uint32_t block;    // resolved CTA size
 };
 
+// The launch configuration of the most recent kernel (sr_last_launch).
+void record_launch(uint32_t grid, uint32_t block, uint32_t smem_bytes);
+
 // Each returns a cudaError_t from the launch (cudaGetLastError after it).
 cudaError_t launch_divloop(const LaunchCtx& c, const sr_workload& w, uint64_t n, uint32_t iters,
                            uint64_t seed, int mode, uint32_t T);
@@ -38,6 +41,9 @@ cudaError_t launch_mcml(const LaunchCtx& c, const sr_workload& w, uint64_t n, ui
                         uint64_t seed, int mode, uint32_t T);
 cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t n,
                              uint32_t iters, uint64_t seed, int mode, uint32_t T);
+
+cudaError_t launch_math_eval(cudaStream_t st, int sm_count, int fn, const float* x, float* out,
+                             uint64_t n);
 
 // Validation of workload-specific parameters; returns "" when fine.
 std::string check_mcml(const sr_mcml_params& p);

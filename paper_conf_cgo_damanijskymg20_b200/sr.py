@@ -26,7 +26,9 @@ SCHED_WORDS = 8
 MC_COUNTERS = ["photons", "steps", "rd_exits", "tt_exits", "rr_kills", "rr_survive", "capped",
                "zero_w"]
 EXPORTS = ["sr_init", "sr_workspace_bytes", "sr_workspace_region", "sr_run", "sr_tally",
-           "sr_finalize", "sr_last_error", "sr_build_info", "sr_scene_build"]
+           "sr_finalize", "sr_last_error", "sr_build_info", "sr_last_launch", "sr_math_eval",
+           "sr_scene_build"]
+FN_LOGF, FN_SIN2PI, FN_COS2PI, FN_EXPENSIVE_1000, FN_EXPENSIVE_2000 = 0, 1, 2, 3, 4
 
 
 class SRError(RuntimeError):
@@ -69,11 +71,13 @@ class Workload(C.Structure):
 _lib = None
 
 
-def load(path: str = LIB_PATH):
-    """Load libsr.so.  Raises FileNotFoundError if it was not built."""
+def load(path: str | None = None):
+    """Load libsr.so (or $SR_LIB, an alternative in-tree build used for
+    tuning experiments).  Raises FileNotFoundError if it was not built."""
     global _lib
     if _lib is not None:
         return _lib
+    path = path or os.environ.get("SR_LIB") or LIB_PATH
     if not os.path.exists(path):
         raise FileNotFoundError(
             f"{path} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'`"
@@ -89,10 +93,13 @@ def load(path: str = LIB_PATH):
     L.sr_finalize.argtypes = []
     L.sr_last_error.restype = C.c_char_p
     L.sr_build_info.restype = C.c_char_p
+    L.sr_last_launch.argtypes = [C.POINTER(C.c_uint32)]
+    L.sr_math_eval.argtypes = [C.c_int, vp, vp, u64]
+    L.sr_math_eval.restype = C.c_int
     fp, up = C.POINTER(C.c_float), C.POINTER(C.c_uint32)
     L.sr_scene_build.argtypes = [fp, up, u32, fp, u32, fp, vp, sz, C.POINTER(sz)]
     for name in ("sr_init", "sr_workspace_region", "sr_run", "sr_tally", "sr_finalize",
-                 "sr_scene_build"):
+                 "sr_last_launch", "sr_scene_build"):
         getattr(L, name).restype = C.c_int
     _lib = L
     return L
@@ -139,6 +146,16 @@ def sr_last_error() -> str:
 
 def sr_build_info() -> str:
     return load().sr_build_info().decode()
+
+
+def sr_math_eval(fn: int, x_ptr: int, out_ptr: int, n: int) -> None:
+    _check(load().sr_math_eval(fn, x_ptr, out_ptr, n))
+
+
+def sr_last_launch() -> dict:
+    out = (C.c_uint32 * 4)()
+    _check(load().sr_last_launch(out))
+    return {"grid": out[0], "block": out[1], "smem": out[2], "kernels": out[3]}
 
 
 def sr_scene_build(tris, mat, mats, cam, dst_ptr: int | None, dst_bytes: int) -> int:

@@ -41,6 +41,33 @@ def run_divloop(ctx, w, n, iters, seed, mode, T):
     return out[:, 0].view(np.float32).copy(), out[:, 1].view(np.uint32).copy(), cnt
 
 
+# ------------------------------------------------------------------ building blocks
+@pytest.mark.parametrize("fn", [sr.FN_LOGF, sr.FN_SIN2PI, sr.FN_COS2PI])
+def test_device_math_bit_exact_all_rng_inputs(ctx, fn):
+    """sr_logf / sr_sincos2pif on every one of the 2^24 inputs the RNG can give."""
+    k = np.arange(1 if fn == sr.FN_LOGF else 0, (1 << 24) + (1 if fn == sr.FN_LOGF else 0),
+                  dtype=np.float64)
+    x = (k * 2.0**-24).astype(np.float32)
+    xd = torch.from_numpy(x).cuda()
+    od = torch.empty_like(xd)
+    sr.sr_math_eval(fn, xd.data_ptr(), od.data_ptr(), x.size)
+    ctx.stream.synchronize()
+    got = od.cpu().numpy()
+    ref = oracle.eval_batch(fn, x)
+    bad = np.nonzero(got.view(np.uint32) != ref.view(np.uint32))[0]
+    assert bad.size == 0, (bad[:5], x[bad[:5]], got[bad[:5]], ref[bad[:5]])
+
+
+@pytest.mark.parametrize("fn", [sr.FN_EXPENSIVE_1000, sr.FN_EXPENSIVE_2000])
+def test_device_expensive_bit_exact(ctx, fn):
+    x = (np.arange(1 << 16, dtype=np.float64) * 2.0**-16).astype(np.float32)
+    xd = torch.from_numpy(x).cuda()
+    od = torch.empty_like(xd)
+    sr.sr_math_eval(fn, xd.data_ptr(), od.data_ptr(), x.size)
+    ctx.stream.synchronize()
+    assert np.array_equal(od.cpu().numpy().view(np.uint32), oracle.eval_batch(fn, x).view(np.uint32))
+
+
 # ------------------------------------------------------------------ config 1
 @pytest.mark.parametrize("seed", SEEDS)
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 4),
