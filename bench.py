@@ -204,6 +204,7 @@ def main():
     import torch.distributed as dist
 
     from paper_conf_cgo_damanijskymg20_b200 import inputs as I
+    from paper_conf_cgo_damanijskymg20_b200 import parallel as P
     from paper_conf_cgo_damanijskymg20_b200 import sr
 
     ws_n, rank, local = dist_env()
@@ -221,7 +222,7 @@ def main():
     per_rank = nt * iters
     T = args.threshold
     w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
-                         task_offset=rank * per_rank)
+                         task_offset=P.task_offset_of(rank, per_rank))
     nbytes = sr.sr_workspace_bytes(w, nt)
     ctx = sr.Context.create(local, nbytes, stream)
     off, tb = sr.sr_workspace_region(w, nt, sr.T_GRID)
@@ -232,9 +233,7 @@ def main():
 
     def step(mode, thr):
         sr.sr_run(w, nt, iters, I.PRIMARY_SEED, mode, thr)
-        if ws_n > 1:
-            with torch.cuda.stream(stream):
-                dist.all_reduce(tallies, op=dist.ReduceOp.SUM)
+        P.allreduce_tallies(tallies, stream=stream)   # no-op at N = 1
 
     # device-timed region, SPEC (headline) with clocks sampled during it
     with ClockSampler(local) as clk:
@@ -281,7 +280,8 @@ def main():
     # schedule-level efficiency of the common code (instrumented kernels, outside timing)
     def region_eff(mode, thr):
         wi = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz,
-                              m.step_cap, task_offset=rank * per_rank, flags=sr.F_SCHED)
+                              m.step_cap, task_offset=P.task_offset_of(rank, per_rank),
+                              flags=sr.F_SCHED)
         ctx.ensure(sr.sr_workspace_bytes(wi, nt))
         ni = min(nt, 32768)
         sr.sr_run(wi, ni, iters, I.PRIMARY_SEED, mode, thr)
