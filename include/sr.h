@@ -181,6 +181,17 @@ enum { SR_FN_LOGF = 0, SR_FN_SIN2PI = 1, SR_FN_COS2PI = 2, SR_FN_EXPENSIVE_1000 
        SR_FN_EXPENSIVE_2000 = 4 };
 SR_API int sr_math_eval(int fn, const float* x_dev, float* out_dev, uint64_t n);
 
+/* Diagnostics: closest hit of n rays against a scene built by sr_scene_build,
+ * with the BVH traversal the PATHTRACE kernels use (reading R7).
+ *   rays_dev  device, n x 6 floats {origin xyz, direction xyz}
+ *   hit_dev   device, n int64: original triangle index (ties -> smaller
+ *             index), -1 = no hit with t > 1e-4
+ *   t_dev     device, n floats: hit distance (+inf on a miss)
+ * On the context stream; no synchronize.  Errors: SR_E_STATE before
+ * sr_init; SR_E_INVALID (NULL arrays with n > 0, not a scene image). */
+SR_API int sr_pt_closest(const void* scene_dev, const float* rays_dev, int64_t* hit_dev,
+                         float* t_dev, uint64_t n);
+
 /* PATHTRACE scene (config 4): build the BVH over a caller-provided triangle
  * soup on the host and write the device scene image.
  *   tris       host, n_tris x 9 floats (v0, v1, v2 xyz), caller-owned

@@ -234,5 +234,47 @@ def ws_divloop_optimum(want):
     return lib().ws_divloop_optimum(_p(want, C.c_uint8), want.shape[0], want.shape[1])
 
 
-def _bind_pt(L):  # filled in by pathtrace support
-    pass
+class PTScene(C.Structure):
+    _fields_ = [("tris", C.POINTER(C.c_float)), ("mat", C.POINTER(C.c_uint32)),
+                ("n_tris", C.c_uint32), ("mats", C.POINTER(C.c_float)), ("n_mats", C.c_uint32),
+                ("cam", C.c_float * 16)]
+
+
+def _bind_pt(L):
+    fp = C.POINTER(C.c_float)
+    L.or_pt_closest.argtypes = [fp, C.c_uint32, fp, fp, fp]
+    L.or_pt_closest.restype = C.c_int64
+    L.or_pt_render.argtypes = [C.POINTER(PTScene), C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32,
+                               C.c_uint64, C.POINTER(C.c_uint32), C.c_uint32, fp,
+                               C.POINTER(C.c_uint64)]
+
+
+def pt_scene(tris, mat, mats, cam):
+    """Keeps the numpy arrays alive alongside the ctypes view."""
+    tris = np.ascontiguousarray(tris, np.float32); mat = np.ascontiguousarray(mat, np.uint32)
+    mats = np.ascontiguousarray(mats, np.float32)
+    s = PTScene(_p(tris, C.c_float), _p(mat, C.c_uint32), len(mat), _p(mats, C.c_float), len(mats))
+    for i, v in enumerate(np.asarray(cam, np.float32)[:16]):
+        s.cam[i] = v
+    s._keep = (tris, mat, mats)
+    return s
+
+
+def pt_render(scene, width, height, spp, max_depth, seed, pixels=None):
+    lib()
+    n = width * height if pixels is None else len(pixels)
+    rgb = np.zeros(3 * n, np.float32)
+    cnt = np.zeros(2, np.uint64)
+    pix = None if pixels is None else np.ascontiguousarray(pixels, np.uint32)
+    lib().or_pt_render(C.byref(scene), width, height, spp, max_depth, seed,
+                       None if pix is None else _p(pix, C.c_uint32), n, _p(rgb, C.c_float),
+                       _p(cnt, C.c_uint64))
+    return rgb.reshape(n, 3), dict(paths=int(cnt[0]), rays=int(cnt[1]))
+
+
+def pt_closest(scene, o, d):
+    o = np.ascontiguousarray(o, np.float32); d = np.ascontiguousarray(d, np.float32)
+    t = C.c_float()
+    i = lib().or_pt_closest(scene.tris, scene.n_tris, _p(o, C.c_float), _p(d, C.c_float),
+                            C.byref(t))
+    return int(i), t.value

@@ -95,6 +95,24 @@ float or_mcml_fresnel(float ni, float nt, float ca1, float* ca2);
 /* Rsp as defined in mcml.c (specular reflectance at launch) */
 float or_mcml_rsp(const or_mcml_params* p);
 
+/* ---- pathtrace.c : config 4, path tracer with brute-force closest hit. */
+typedef struct {
+  const float* tris;     /* n_tris x 9 floats (v0, v1, v2)                  */
+  const uint32_t* mat;   /* n_tris material ids                             */
+  uint32_t n_tris;
+  const float* mats;     /* n_mats x 8 {kind, r, g, b, er, eg, eb, ior}     */
+  uint32_t n_mats;
+  float cam[16];         /* eye, forward, right, up, tan(fov/2), aspect     */
+} or_pt_scene;
+/* closest hit over all triangles (t > 1e-4; ties -> smaller index); -1 = miss */
+int64_t or_pt_closest(const float* tris, uint32_t n_tris, const float o[3], const float d[3],
+                      float* t_best);
+/* rgb[3k..3k+2] = sum over the spp samples of pixel pixels[k] (all pixels
+ * 0..n_pixels-1 when pixels == NULL); counters[0] += paths, [1] += rays. */
+void or_pt_render(const or_pt_scene* sc, uint32_t width, uint32_t height, uint32_t spp,
+                  uint32_t max_depth, uint64_t seed, const uint32_t* pixels, uint32_t n_pixels,
+                  float* rgb, uint64_t* counters);
+
 /* ---- warpsim.c : lane-mask warp simulator (oracle part 2). */
 enum { WS_PDOM = 0, WS_SPEC_LOOP = 1, WS_SPEC_CALL = 2 };
 /* regions of the divloop program (Listing 1) */

@@ -1,20 +1,461 @@
-// pathtrace.cu -- config 4 (path tracer, Loop Merge over bounces).
-// Placeholder until the path tracer lands: the ABI rejects the workload.
+// pathtrace.cu -- config 4: path tracer over a BVH scene (the paper's
+// "pathtracer", Table 2; Russian roulette and bounded bounces,
+// P:1377-1383), Loop Merge over the bounce loop (Fig. 2(b)), the
+// samples per pixel being the coarsened outer loop:
+//
+//   for (s = 0; s < spp; s++) {                  // outer loop
+//     Prolog: camera ray of sample s
+//     for (b = 0; alive; b++) { L1: bounce() }   // divergent trip count
+//     Epilog: pixel += radiance
+//   }
+//
+//   pt_pdom  as written: a warp's 32 pixels trace sample s together; lanes
+//            whose path ended idle until the longest path of the warp ends.
+//   pt_spec  Loop Merge + soft barrier: P = ballot(path in flight); if
+//            popc(P) >= T or no idle lane has a sample left, every in-flight
+//            lane takes one bounce; otherwise idle lanes run the epilog and
+//            the next camera ray.  "PathTracer executes fastest when all
+//            threads reconverge" -> default T = 32.
+//
+// One lane = one pixel (static; the pixel sum is accumulated in sample order,
+// so the float result is schedule-free).  bounce() = BVH closest hit (exactly
+// the brute-force closest hit, ties to the smaller triangle id; conservative
+// padded-box slab test) + material shading, operation for operation as
+// oracle/pathtrace.c (reading R7).
+#include "pt_scene.h"
+#include "sr_device.cuh"
 #include "sr_internal.h"
 
 namespace sr {
-std::string check_pathtrace(const sr_pathtrace_params&, uint64_t) {
-  return "SR_WL_PATHTRACE is not implemented in this build";
-}
-size_t pathtrace_perthread_bytes(uint64_t n) { return 12 * n; }
-cudaError_t launch_pathtrace(const LaunchCtx&, const sr_workload&, uint64_t, uint32_t, uint64_t,
-                             int, uint32_t) {
-  return cudaErrorNotSupported;
-}
-}  // namespace sr
+namespace {
 
-extern "C" int sr_scene_build(const float*, const uint32_t*, uint32_t, const float*, uint32_t,
-                              const float*, void*, size_t, size_t* needed) {
-  if (needed) *needed = 0;
-  return SR_E_INVALID;
+constexpr float kTmin = 1.0e-4f;
+constexpr float kDetEps = 1.0e-12f;
+constexpr int kStack = 64;  // > BVH depth (binned SAH over 1M triangles: ~40)
+
+struct V3 {
+  float x, y, z;
+};
+__device__ __forceinline__ V3 mk(float x, float y, float z) { return {x, y, z}; }
+__device__ __forceinline__ V3 sub(V3 a, V3 b) { return mk(a.x - b.x, a.y - b.y, a.z - b.z); }
+__device__ __forceinline__ V3 add(V3 a, V3 b) { return mk(a.x + b.x, a.y + b.y, a.z + b.z); }
+__device__ __forceinline__ V3 scl(V3 a, float s) { return mk(a.x * s, a.y * s, a.z * s); }
+__device__ __forceinline__ float dot(V3 a, V3 b) { return (a.x * b.x + a.y * b.y) + a.z * b.z; }
+__device__ __forceinline__ V3 cross(V3 a, V3 b) {
+  return mk(a.y * b.z - a.z * b.y, a.z * b.x - a.x * b.z, a.x * b.y - a.y * b.x);
 }
+__device__ __forceinline__ V3 normalize(V3 a) {
+  const float inv = 1.0f / sqrtf(dot(a, a));
+  return scl(a, inv);
+}
+
+struct PtArgs {
+  const unsigned char* scene;
+  const PtNode* nodes;
+  const PtTri* tris;
+  const PtMat* mats;
+  uint32_t width, height, spp, max_depth, T;
+  uint64_t n, seed;
+  float* rgb;                       // 3 floats per pixel
+  unsigned long long* counters;     // [0] paths [1] rays [2] node visits [3] tri tests
+  uint32_t* sched;
+  // diagnostics (sr_pt_closest): rays in, hits out
+  const float* q_rays;
+  int64_t* q_hit;
+  float* q_t;
+};
+
+struct Stats {
+  uint32_t rays, nodes, tests;
+};
+
+// Conservative slab test against a padded box: accept when the ray's
+// parametric interval [tmin, tbest] can touch the box (slack 1e-5 relative).
+__device__ __forceinline__ bool box_hit(const float* lo, const float* hi, V3 o, V3 inv, float tb,
+                                        float& tnear) {
+  const float tx0 = (lo[0] - o.x) * inv.x, tx1 = (hi[0] - o.x) * inv.x;
+  const float ty0 = (lo[1] - o.y) * inv.y, ty1 = (hi[1] - o.y) * inv.y;
+  const float tz0 = (lo[2] - o.z) * inv.z, tz1 = (hi[2] - o.z) * inv.z;
+  const float tn = fmaxf(fmaxf(fminf(tx0, tx1), fminf(ty0, ty1)), fmaxf(fminf(tz0, tz1), 0.0f));
+  const float tf = fminf(fminf(fmaxf(tx0, tx1), fmaxf(ty0, ty1)), fmaxf(tz0, tz1));
+  tnear = tn;
+  return tn * (1.0f - 1e-5f) <= tf * (1.0f + 1e-5f) && tn * (1.0f - 1e-5f) <= tb;
+}
+
+// Moller-Trumbore exactly as the oracle (e1, e2 precomputed with the same
+// binary32 subtractions).
+__device__ __forceinline__ void tri_test(const PtTri& T, V3 o, V3 d, float& tb, int64_t& ib,
+                                         uint32_t& mb) {
+  const V3 v0 = mk(T.v0[0], T.v0[1], T.v0[2]);
+  const V3 e1 = mk(T.e1[0], T.e1[1], T.e1[2]);
+  const V3 e2 = mk(T.e2[0], T.e2[1], T.e2[2]);
+  const V3 pv = cross(d, e2);
+  const float det = dot(e1, pv);
+  if (fabsf(det) < kDetEps) return;
+  const float inv = 1.0f / det;
+  const V3 tv = sub(o, v0);
+  const float u = dot(tv, pv) * inv;
+  if (u < 0.0f || u > 1.0f) return;
+  const V3 qv = cross(tv, e1);
+  const float v = dot(d, qv) * inv;
+  if (v < 0.0f || u + v > 1.0f) return;
+  const float t = dot(e2, qv) * inv;
+  if (!(t > kTmin)) return;
+  const int64_t id = (int64_t)T.id;
+  if (t < tb || (t == tb && id < ib)) {   // ties -> smaller original id (= brute force)
+    tb = t;
+    ib = id;
+    mb = T.mat;
+  }
+}
+
+__device__ int64_t closest_hit(const PtArgs& a, V3 o, V3 d, float& t_out, uint32_t& mat_out,
+                               uint32_t& tri_slot, Stats& st) {
+  const V3 inv = mk(1.0f / d.x, 1.0f / d.y, 1.0f / d.z);
+  float tb = INFINITY;
+  int64_t ib = -1;
+  uint32_t mb = 0;
+  int32_t stack[kStack];
+  int sp = 0;
+  int32_t node = 0;
+  uint32_t slot = 0;
+  for (;;) {
+    const PtNode N = a.nodes[node];
+    ++st.nodes;
+    float tn0, tn1;
+    const bool h0 = N.cnt0 >= 0 && N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, inv, tb, tn0);
+    const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, o, inv, tb, tn1);
+    int32_t next = -1;
+    // leaves: test their triangles now; inner children: descend / push
+    if (h0 && N.cnt0 > 0) {
+      for (int32_t k = 0; k < N.cnt0; ++k) {
+        const int64_t before = ib;
+        tri_test(a.tris[N.ref0 + k], o, d, tb, ib, mb);
+        if (ib != before) slot = (uint32_t)(N.ref0 + k);
+        ++st.tests;
+      }
+    }
+    if (h1 && N.cnt1 > 0) {
+      for (int32_t k = 0; k < N.cnt1; ++k) {
+        const int64_t before = ib;
+        tri_test(a.tris[N.ref1 + k], o, d, tb, ib, mb);
+        if (ib != before) slot = (uint32_t)(N.ref1 + k);
+        ++st.tests;
+      }
+    }
+    const bool in0 = h0 && N.cnt0 == 0, in1 = h1 && N.cnt1 == 0;
+    if (in0 && in1) {
+      const bool first0 = tn0 <= tn1;
+      next = first0 ? N.ref0 : N.ref1;
+      if (sp < kStack) stack[sp++] = first0 ? N.ref1 : N.ref0;
+    } else if (in0) {
+      next = N.ref0;
+    } else if (in1) {
+      next = N.ref1;
+    }
+    if (next < 0) {
+      if (sp == 0) break;
+      next = stack[--sp];
+    }
+    node = next;
+  }
+  t_out = tb;
+  mat_out = mb;
+  tri_slot = slot;
+  return ib;
+}
+
+struct Path {
+  V3 o, d, thr, rad, sum;
+  uint32_t pix, s, b;
+  bool alive;
+};
+
+__device__ __forceinline__ void camera_ray(const PtArgs& a, const PtHeader& H, Path& p) {
+  const uint64_t q = (uint64_t)p.pix * a.spp + p.s;
+  const uint4 u = draw(0u, kTagPt, q, a.seed);
+  const uint32_t px = p.pix % a.width, py = p.pix / a.width;
+  const float fx = ((float)px + u01(u.x)) / (float)a.width;
+  const float fy = ((float)py + u01(u.y)) / (float)a.height;
+  const float tan_half = H.cam[12], aspect = H.cam[13];
+  const float sx = (2.0f * fx - 1.0f) * tan_half * aspect;
+  const float sy = (1.0f - 2.0f * fy) * tan_half;
+  const V3 fwd = mk(H.cam[3], H.cam[4], H.cam[5]);
+  const V3 right = mk(H.cam[6], H.cam[7], H.cam[8]);
+  const V3 up = mk(H.cam[9], H.cam[10], H.cam[11]);
+  p.d = normalize(add(add(fwd, scl(right, sx)), scl(up, sy)));
+  p.o = mk(H.cam[0], H.cam[1], H.cam[2]);
+  p.thr = mk(1.0f, 1.0f, 1.0f);
+  p.rad = mk(0.0f, 0.0f, 0.0f);
+  p.b = 0;
+  p.alive = true;
+}
+
+__device__ __forceinline__ void onb(V3 n, V3& t1, V3& t2) {
+  const float sign = copysignf(1.0f, n.z);
+  const float a = -1.0f / (sign + n.z);
+  const float b = n.x * n.y * a;
+  t1 = mk(1.0f + sign * n.x * n.x * a, sign * b, -sign * n.x);
+  t2 = mk(b, sign + n.y * n.y * a, -n.y);
+}
+
+// One bounce (the common inner-loop body).  Ends the path when it escapes,
+// hits a light, reaches max_depth or loses the roulette; the epilog (pixel
+// sum) happens at that point, in sample order.
+__device__ void bounce(const PtArgs& a, Path& p, Stats& st) {
+  float t;
+  uint32_t mat, slot;
+  const int64_t hit = closest_hit(a, p.o, p.d, t, mat, slot, st);
+  ++st.rays;
+  bool end = hit < 0;
+  if (!end) {
+    const PtMat m = a.mats[mat];
+    const uint32_t kind = (uint32_t)m.kind;
+    p.rad = add(p.rad, mk(p.thr.x * m.er, p.thr.y * m.eg, p.thr.z * m.eb));
+    if (kind == 3u) {
+      end = true;
+    } else {
+      const PtTri& T = a.tris[slot];
+      const V3 e1 = mk(T.e1[0], T.e1[1], T.e1[2]);
+      const V3 e2 = mk(T.e2[0], T.e2[1], T.e2[2]);
+      const V3 ng = normalize(cross(e1, e2));
+      const float cosd = dot(ng, p.d);
+      const bool entering = cosd < 0.0f;
+      const V3 n = entering ? ng : scl(ng, -1.0f);
+      const V3 pt = add(p.o, scl(p.d, t));
+      const uint64_t q = (uint64_t)p.pix * a.spp + p.s;
+      const uint4 u = draw(p.b + 1u, kTagPt, q, a.seed);
+      if (kind == 0u) {
+        const float r1 = u01(u.x);
+        const float rr = sqrtf(r1);
+        float sp, cp;
+        sr_sincos2pif(u01(u.y), sp, cp);
+        const float lx = rr * cp, ly = rr * sp, lz = sqrtf(1.0f - r1);
+        V3 t1, t2;
+        onb(n, t1, t2);
+        p.d = add(add(scl(t1, lx), scl(t2, ly)), scl(n, lz));
+      } else if (kind == 1u) {
+        p.d = sub(p.d, scl(n, 2.0f * dot(p.d, n)));
+      } else {
+        const float ior = m.ior;
+        const float eta = entering ? 1.0f / ior : ior;
+        const float cosi = -dot(p.d, n);
+        const float k = 1.0f - eta * eta * (1.0f - cosi * cosi);
+        float r0 = (1.0f - ior) / (1.0f + ior);
+        r0 = r0 * r0;
+        const float c5 = 1.0f - cosi;
+        const float fr = r0 + (1.0f - r0) * (c5 * c5 * c5 * c5 * c5);
+        if (k < 0.0f || u01(u.z) < fr) p.d = sub(p.d, scl(n, 2.0f * dot(p.d, n)));
+        else p.d = add(scl(p.d, eta), scl(n, eta * cosi - sqrtf(k)));
+      }
+      p.thr = mk(p.thr.x * m.r, p.thr.y * m.g, p.thr.z * m.b);
+      p.o = pt;
+      if (p.b >= 3u) {
+        const float pm = fmaxf(p.thr.x, fmaxf(p.thr.y, p.thr.z));
+        const float prr = fminf(0.95f, pm);
+        if (!(u01(u.w) < prr)) end = true;
+        else p.thr = mk(p.thr.x / prr, p.thr.y / prr, p.thr.z / prr);
+      }
+    }
+  }
+  p.b = p.b + 1u;
+  if (!end && p.b >= a.max_depth) end = true;
+  if (end) {
+    p.sum = add(p.sum, p.rad);   // Epilog: pixel += radiance (sample order)
+    p.alive = false;
+  }
+}
+
+__device__ __forceinline__ void finish(const PtArgs& a, const Path& p, bool valid, Stats st,
+                                       uint32_t paths, uint64_t warp, uint32_t rounds,
+                                       uint32_t rel, uint32_t rel_lanes, uint32_t adv,
+                                       uint32_t adv_lanes) {
+  if (valid) {
+    a.rgb[3 * (uint64_t)p.pix + 0] = p.sum.x;
+    a.rgb[3 * (uint64_t)p.pix + 1] = p.sum.y;
+    a.rgb[3 * (uint64_t)p.pix + 2] = p.sum.z;
+  }
+  unsigned long long v[4] = {paths, st.rays, st.nodes, st.tests};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v[i] += __shfl_xor_sync(kFull, v[i], o);
+  }
+  if (lane_id() == 0) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) atomicAdd(&a.counters[i], v[i]);
+    if (a.sched) {
+      uint4* s = reinterpret_cast<uint4*>(a.sched + warp * kSchedWords);
+      s[0] = make_uint4(rounds, rel, rel_lanes, adv);
+      s[1] = make_uint4(adv_lanes, 0u, 0u, 0u);
+    }
+  }
+}
+
+template <bool SCHED>
+__global__ void __launch_bounds__(128) pt_pdom(const PtArgs a) {
+  const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
+  const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const bool valid = g < a.n;
+  Path p;
+  p.pix = (uint32_t)(valid ? g : 0);
+  p.sum = mk(0.0f, 0.0f, 0.0f);
+  p.alive = false;
+  Stats st{0, 0, 0};
+  uint32_t paths = 0, outer = 0, rel = 0, rel_lanes = 0, launch_lanes = 0;
+  for (uint32_t s = 0; s < a.spp; ++s) {
+    if (SCHED) { ++outer; launch_lanes += __popc(__ballot_sync(kFull, valid)); }
+    if (valid) {
+      p.s = s;
+      camera_ray(a, H, p);              // Prolog
+      ++paths;
+      do {                              // L1: bounce loop, divergent trip count
+        if constexpr (SCHED) {
+          const uint32_t m = __activemask();
+          if (lane_id() == (uint32_t)(__ffs(m) - 1)) { ++rel; rel_lanes += __popc(m); }
+        }
+        bounce(a, p, st);
+      } while (p.alive);
+    }                                   // IPDOM: reconverge, next sample
+  }
+  uint32_t r = 0, rl = 0;
+  if constexpr (SCHED) { r = __reduce_add_sync(kFull, rel); rl = __reduce_add_sync(kFull, rel_lanes); }
+  finish(a, p, valid, st, paths, g >> 5, outer, r, rl, outer, launch_lanes);
+}
+
+template <bool SCHED>
+__global__ void __launch_bounds__(128) pt_spec(const PtArgs a) {
+  const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
+  const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const bool valid = g < a.n;
+  Path p;
+  p.pix = (uint32_t)(valid ? g : 0);
+  p.sum = mk(0.0f, 0.0f, 0.0f);
+  p.alive = false;
+  p.s = 0;
+  Stats st{0, 0, 0};
+  uint32_t paths = 0, rounds = 0, rel = 0, rel_lanes = 0, adv = 0, adv_lanes = 0;
+  uint32_t next_s = 0;
+  uint32_t E = __ballot_sync(kFull, !valid || a.spp == 0);  // lanes with no sample left
+  for (;;) {
+    const uint32_t P = __ballot_sync(kFull, p.alive);
+    const uint32_t R = ~(P | E);
+    if ((P | R) == 0u) break;
+    if constexpr (SCHED) ++rounds;
+    if ((uint32_t)__popc(P) >= a.T || R == 0u) {
+      if constexpr (SCHED) { ++rel; rel_lanes += __popc(P); }
+      if (p.alive) {
+        __syncwarp(P);
+        bounce(a, p, st);
+      }
+    } else {
+      if constexpr (SCHED) { ++adv; adv_lanes += __popc(R); }
+      if ((R >> lane_id()) & 1u) {
+        p.s = next_s++;
+        camera_ray(a, H, p);
+        ++paths;
+      }
+      E = __ballot_sync(kFull, !valid || next_s >= a.spp);  // no sample left to start
+    }
+  }
+  finish(a, p, valid, st, paths, g >> 5, rounds, rel, rel_lanes, adv, adv_lanes);
+}
+
+// sr_pt_closest diagnostics: one ray per thread
+__global__ void pt_query(const PtArgs a) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= a.n) return;
+  const float* r = a.q_rays + 6 * i;
+  Stats st{0, 0, 0};
+  float t;
+  uint32_t mat, slot;
+  const int64_t h = closest_hit(a, mk(r[0], r[1], r[2]), mk(r[3], r[4], r[5]), t, mat, slot, st);
+  a.q_hit[i] = h;
+  a.q_t[i] = t;
+}
+
+PtArgs base_args(const void* scene) {
+  PtArgs a{};
+  const unsigned char* s = static_cast<const unsigned char*>(scene);
+  a.scene = s;
+  // header offsets are read on the host from a copy (see check_pathtrace)
+  return a;
+}
+
+}  // namespace
+
+std::string check_pathtrace(const sr_pathtrace_params& p, uint64_t n_threads) {
+  if (!p.scene_dev) return "pathtrace.scene_dev is NULL (build it with sr_scene_build)";
+  if (p.scene_bytes < sizeof(PtHeader)) return "pathtrace.scene_bytes too small";
+  if (p.width == 0 || p.height == 0) return "pathtrace.width/height must be >= 1";
+  if ((uint64_t)p.width * p.height != n_threads)
+    return "pathtrace: n_threads must equal width*height (one lane per pixel)";
+  if (p.max_depth == 0) return "pathtrace.max_depth must be >= 1";
+  return "";
+}
+
+size_t pathtrace_perthread_bytes(uint64_t n) { return 12 * n; }
+
+static cudaError_t read_header(const void* scene, PtHeader& h) {
+  cudaError_t e = cudaMemcpy(&h, scene, sizeof h, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return e;
+  if (h.magic != kPtMagic) return cudaErrorInvalidValue;
+  return cudaSuccess;
+}
+
+cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t n, uint32_t iters,
+                             uint64_t seed, int mode, uint32_t T) {
+  PtHeader h;
+  cudaError_t e = read_header(w.pathtrace.scene_dev, h);
+  if (e != cudaSuccess) return e;
+  if (h.bytes > w.pathtrace.scene_bytes) return cudaErrorInvalidValue;
+  PtArgs a = base_args(w.pathtrace.scene_dev);
+  a.nodes = reinterpret_cast<const PtNode*>(a.scene + h.off_nodes);
+  a.tris = reinterpret_cast<const PtTri*>(a.scene + h.off_tris);
+  a.mats = reinterpret_cast<const PtMat*>(a.scene + h.off_mats);
+  a.width = w.pathtrace.width;
+  a.height = w.pathtrace.height;
+  a.spp = iters;
+  a.max_depth = w.pathtrace.max_depth;
+  a.T = T;
+  a.n = n;
+  a.seed = seed;
+  a.rgb = reinterpret_cast<float*>(c.ws + c.lay.off[SR_T_PERTHREAD]);
+  a.counters = reinterpret_cast<unsigned long long*>(c.ws + c.lay.off[SR_T_COUNTERS]);
+  a.sched = (w.flags & SR_F_SCHED) ? reinterpret_cast<uint32_t*>(c.ws + c.lay.off[SR_T_SCHED])
+                                   : nullptr;
+  const uint32_t block = c.block;
+  const uint64_t grid = (n + block - 1) / block;
+  if (grid > 0x7fffffffull) return cudaErrorInvalidConfiguration;
+  record_launch((uint32_t)grid, block, 0);
+  const bool spec = mode == SR_SPEC_LOOP;
+  if (a.sched) {
+    if (spec) pt_spec<true><<<(unsigned)grid, block, 0, c.stream>>>(a);
+    else pt_pdom<true><<<(unsigned)grid, block, 0, c.stream>>>(a);
+  } else {
+    if (spec) pt_spec<false><<<(unsigned)grid, block, 0, c.stream>>>(a);
+    else pt_pdom<false><<<(unsigned)grid, block, 0, c.stream>>>(a);
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* rays, int64_t* hit,
+                            float* t, uint64_t n) {
+  PtHeader h;
+  cudaError_t e = read_header(scene, h);
+  if (e != cudaSuccess) return e;
+  PtArgs a = base_args(scene);
+  a.nodes = reinterpret_cast<const PtNode*>(a.scene + h.off_nodes);
+  a.tris = reinterpret_cast<const PtTri*>(a.scene + h.off_tris);
+  a.mats = reinterpret_cast<const PtMat*>(a.scene + h.off_mats);
+  a.n = n;
+  a.q_rays = rays;
+  a.q_hit = hit;
+  a.q_t = t;
+  const unsigned grid = (unsigned)((n + 127) / 128);
+  record_launch(grid, 128, 0);
+  if (n) pt_query<<<grid, 128, 0, st>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace sr

@@ -79,6 +79,8 @@ uint32_t default_block(const sr_workload& w) {
 
 }  // namespace
 
+int set_error(int code, const std::string& msg) { return fail(code, msg); }
+
 void record_launch(uint32_t grid, uint32_t block, uint32_t smem_bytes) {
   g_launch[0] = grid;
   g_launch[1] = block;
@@ -148,6 +150,19 @@ int sr_math_eval(int fn, const float* x_dev, float* out_dev, uint64_t n) {
   if (!n) return SR_OK;
   const cudaError_t e = launch_math_eval(g_ctx.stream, g_ctx.sm_count, fn, x_dev, out_dev, n);
   if (e != cudaSuccess) return fail_cuda(e, "sr_math_eval");
+  return SR_OK;
+}
+
+int sr_pt_closest(const void* scene_dev, const float* rays_dev, int64_t* hit_dev, float* t_dev,
+                  uint64_t n) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  g_err.clear();
+  if (!scene_dev || (n && (!rays_dev || !hit_dev || !t_dev)))
+    return fail(SR_E_INVALID, "NULL array");
+  if (!g_ctx.live) return fail(SR_E_STATE, "sr_pt_closest before sr_init");
+  const cudaError_t e = launch_pt_query(g_ctx.stream, scene_dev, rays_dev, hit_dev, t_dev, n);
+  if (e == cudaErrorInvalidValue) return fail(SR_E_INVALID, "scene_dev is not a scene image");
+  if (e != cudaSuccess) return fail_cuda(e, "sr_pt_closest");
   return SR_OK;
 }
 

@@ -29,6 +29,9 @@ struct LaunchCtx {
   uint32_t block;    // resolved CTA size
 };
 
+// Set the calling thread's sr_last_error() text; returns `code`.
+int set_error(int code, const std::string& msg);
+
 // The launch configuration of the most recent kernel (sr_last_launch).
 void record_launch(uint32_t grid, uint32_t block, uint32_t smem_bytes);
 
@@ -44,6 +47,8 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
 
 cudaError_t launch_math_eval(cudaStream_t st, int sm_count, int fn, const float* x, float* out,
                              uint64_t n);
+cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* rays, int64_t* hit,
+                            float* t, uint64_t n);
 
 // Validation of workload-specific parameters; returns "" when fine.
 std::string check_mcml(const sr_mcml_params& p);

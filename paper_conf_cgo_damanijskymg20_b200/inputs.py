@@ -70,3 +70,124 @@ VAN_DE_HULST = MCML(layers=((1.0, 10.0, 90.0, 0.75, 0.02),))
 C1 = DivLoop()
 C2 = CommonCall()
 C3 = MCML()
+
+
+# ---------------------------------------------------------------- config 4 scene
+# Materials: (kind, r, g, b, er, eg, eb, ior); kind 0 diffuse, 1 mirror,
+# 2 dielectric, 3 emissive-only (light).
+MAT_DIFFUSE, MAT_MIRROR, MAT_GLASS, MAT_LIGHT = 0, 1, 2, 3
+
+
+@dataclass(frozen=True)
+class PathTrace:
+    """Config 4 (BASELINE.json configs[3]): Cornell box + icospheres, BVH."""
+    width: int = 1024
+    height: int = 1024
+    spp: int = 16
+    max_depth: int = 8
+    n_spheres: int = 51
+    subdiv: int = 5          # 20 * 4^5 = 20480 triangles per sphere; 51 -> 1,044,494 total
+    fov_deg: float = 65.0
+    scene_seed: int = 20200222
+    threshold: int = 32
+
+    @property
+    def n_pixels(self) -> int:
+        return self.width * self.height
+
+
+C4 = PathTrace()
+C4_SMALL = PathTrace(width=64, height=48, spp=4, subdiv=1)   # oracle-sized parity case
+
+
+def _icosphere(subdiv: int):
+    """Unit icosphere as a float64 triangle soup [n, 3, 3]; midpoints are
+    computed from the two endpoint values only, so shared edges stay shared."""
+    import numpy as np
+    t = (1.0 + 5.0 ** 0.5) / 2.0
+    v = np.array([[-1, t, 0], [1, t, 0], [-1, -t, 0], [1, -t, 0], [0, -1, t], [0, 1, t],
+                  [0, -1, -t], [0, 1, -t], [t, 0, -1], [t, 0, 1], [-t, 0, -1], [-t, 0, 1]],
+                 np.float64)
+    v /= np.linalg.norm(v, axis=1, keepdims=True)
+    f = np.array([[0, 11, 5], [0, 5, 1], [0, 1, 7], [0, 7, 10], [0, 10, 11], [1, 5, 9],
+                  [5, 11, 4], [11, 10, 2], [10, 7, 6], [7, 1, 8], [3, 9, 4], [3, 4, 2],
+                  [3, 2, 6], [3, 6, 8], [3, 8, 9], [4, 9, 5], [2, 4, 11], [6, 2, 10],
+                  [8, 6, 7], [9, 8, 1]])
+    tri = v[f]                                           # [20, 3, 3]
+    for _ in range(subdiv):
+        a, b, c = tri[:, 0], tri[:, 1], tri[:, 2]
+        ab, bc, ca = (a + b), (b + c), (c + a)
+        ab /= np.linalg.norm(ab, axis=1, keepdims=True)
+        bc /= np.linalg.norm(bc, axis=1, keepdims=True)
+        ca /= np.linalg.norm(ca, axis=1, keepdims=True)
+        tri = np.stack([np.stack([a, ab, ca], 1), np.stack([ab, b, bc], 1),
+                        np.stack([ca, bc, c], 1), np.stack([ab, bc, ca], 1)], 1).reshape(-1, 3, 3)
+    return tri
+
+
+def _quad(p0, p1, p2, p3):
+    """Two triangles of the quad p0-p1-p2-p3 (counter-clockwise)."""
+    import numpy as np
+    return np.array([[p0, p1, p2], [p0, p2, p3]], np.float64)
+
+
+def cornell_scene(cfg: PathTrace = C4):
+    """Seeded synthetic scene.  Returns (tris float32 [n, 9], mat uint32 [n],
+    mats float32 [m, 8], cam float32 [12]).
+
+    Closed unit Cornell box with the camera just inside its front wall, a small
+    emissive ceiling quad, and cfg.n_spheres non-overlapping icospheres: 50 % diffuse, 20 %
+    mirror, 20 % glass (ior 1.5), 10 % emissive.  cam = {eye, forward, right,
+    up, tan(fov/2), aspect, 0} as floats (an orthonormal basis, float64 -> f32).
+    """
+    import numpy as np
+    rng = np.random.default_rng(cfg.scene_seed)
+    mats = [(MAT_DIFFUSE, .73, .73, .73, 0, 0, 0, 1.0),   # 0 white walls
+            (MAT_DIFFUSE, .65, .05, .05, 0, 0, 0, 1.0),   # 1 red wall
+            (MAT_DIFFUSE, .12, .45, .15, 0, 0, 0, 1.0),   # 2 green wall
+            (MAT_LIGHT, 0, 0, 0, 15.0, 15.0, 15.0, 1.0)]  # 3 ceiling light
+    tris, mat = [], []
+
+    def add(t, m):
+        tris.append(t)
+        mat.extend([m] * len(t))
+    add(_quad([0, 0, 0], [1, 0, 0], [1, 0, 1], [0, 0, 1]), 0)          # floor
+    add(_quad([0, 1, 0], [0, 1, 1], [1, 1, 1], [1, 1, 0]), 0)          # ceiling
+    add(_quad([0, 0, 1], [1, 0, 1], [1, 1, 1], [0, 1, 1]), 0)          # back
+    add(_quad([0, 0, 0], [0, 1, 0], [1, 1, 0], [1, 0, 0]), 0)          # front (behind camera)
+    add(_quad([0, 0, 0], [0, 0, 1], [0, 1, 1], [0, 1, 0]), 1)          # left, red
+    add(_quad([1, 0, 0], [1, 1, 0], [1, 1, 1], [1, 0, 1]), 2)          # right, green
+    add(_quad([.4, .999, .4], [.4, .999, .6], [.6, .999, .6], [.6, .999, .4]), 3)  # light
+    unit = _icosphere(cfg.subdiv)
+    centres = []
+    kinds = rng.permutation([MAT_DIFFUSE] * 50 + [MAT_MIRROR] * 20 + [MAT_GLASS] * 20 +
+                            [MAT_LIGHT] * 10)
+    while len(centres) < cfg.n_spheres:
+        r = rng.uniform(0.035, 0.075)
+        c = rng.uniform(r + 0.01, 1 - r - 0.01, 3)
+        c[2] = max(c[2], 0.25 + r)          # keep the spheres off the camera
+        if all(np.linalg.norm(c - c2) > r + r2 + 0.005 for c2, r2 in centres):
+            centres.append((c, r))
+    for i, (c, r) in enumerate(centres):
+        kind = int(kinds[i % len(kinds)])
+        col = rng.uniform(0.2, 0.9, 3)
+        if kind == MAT_LIGHT:
+            mats.append((MAT_LIGHT, 0, 0, 0, *(4.0 * col), 1.0))
+        elif kind == MAT_GLASS:
+            mats.append((MAT_GLASS, 1, 1, 1, 0, 0, 0, 1.5))
+        elif kind == MAT_MIRROR:
+            mats.append((MAT_MIRROR, *(0.5 + 0.5 * col), 0, 0, 0, 1.0))
+        else:
+            mats.append((MAT_DIFFUSE, *col, 0, 0, 0, 1.0))
+        add(unit * r + c, len(mats) - 1)
+    tris = np.concatenate(tris).reshape(-1, 9).astype(np.float32)
+    mat = np.array(mat, np.uint32)
+    eye = np.array([0.5, 0.5, 0.02])
+    fwd = np.array([0.5, 0.5, 0.5]) - eye
+    fwd /= np.linalg.norm(fwd)
+    right = np.cross(np.array([0.0, 1.0, 0.0]), fwd)
+    right /= np.linalg.norm(right)
+    up = np.cross(fwd, right)
+    cam = np.concatenate([eye, fwd, right, up,
+                          [np.tan(np.radians(cfg.fov_deg) / 2), cfg.width / cfg.height, 0.0]])
+    return tris, mat, np.array(mats, np.float32), cam.astype(np.float32)

@@ -27,7 +27,8 @@ MC_COUNTERS = ["photons", "steps", "rd_exits", "tt_exits", "rr_kills", "rr_survi
                "zero_w"]
 EXPORTS = ["sr_init", "sr_workspace_bytes", "sr_workspace_region", "sr_run", "sr_tally",
            "sr_finalize", "sr_last_error", "sr_build_info", "sr_last_launch", "sr_math_eval",
-           "sr_scene_build"]
+           "sr_pt_closest", "sr_scene_build"]
+PT_COUNTERS = ["paths", "rays", "node_visits", "tri_tests"]
 FN_LOGF, FN_SIN2PI, FN_COS2PI, FN_EXPENSIVE_1000, FN_EXPENSIVE_2000 = 0, 1, 2, 3, 4
 
 
@@ -96,6 +97,8 @@ def load(path: str | None = None):
     L.sr_last_launch.argtypes = [C.POINTER(C.c_uint32)]
     L.sr_math_eval.argtypes = [C.c_int, vp, vp, u64]
     L.sr_math_eval.restype = C.c_int
+    L.sr_pt_closest.argtypes = [vp, vp, vp, vp, u64]
+    L.sr_pt_closest.restype = C.c_int
     fp, up = C.POINTER(C.c_float), C.POINTER(C.c_uint32)
     L.sr_scene_build.argtypes = [fp, up, u32, fp, u32, fp, vp, sz, C.POINTER(sz)]
     for name in ("sr_init", "sr_workspace_region", "sr_run", "sr_tally", "sr_finalize",
@@ -152,6 +155,10 @@ def sr_math_eval(fn: int, x_ptr: int, out_ptr: int, n: int) -> None:
     _check(load().sr_math_eval(fn, x_ptr, out_ptr, n))
 
 
+def sr_pt_closest(scene_ptr: int, rays_ptr: int, hit_ptr: int, t_ptr: int, n: int) -> None:
+    _check(load().sr_pt_closest(scene_ptr, rays_ptr, hit_ptr, t_ptr, n))
+
+
 def sr_last_launch() -> dict:
     out = (C.c_uint32 * 4)()
     _check(load().sr_last_launch(out))
@@ -196,6 +203,23 @@ def mcml_workload(layers, n_above=1.0, n_below=1.0, dr=0.01, dz=0.002, nr=256, n
     m.n_above, m.n_below, m.dr, m.dz = n_above, n_below, dr, dz
     m.nr, m.nz, m.step_cap = nr, nz, step_cap
     w.mcml = m
+    return w
+
+
+def upload_scene(tris, mat, mats, cam, device: int = 0):
+    """Build the BVH scene image (sr_scene_build) into a torch-owned device
+    buffer; returns (buffer, bytes)."""
+    import torch
+    need = sr_scene_build(tris, mat, mats, cam, None, 0)
+    buf = torch.empty(need, dtype=torch.uint8, device=f"cuda:{device}")
+    used = sr_scene_build(tris, mat, mats, cam, buf.data_ptr(), need)
+    return buf, used
+
+
+def pathtrace_workload(scene_ptr: int, scene_bytes: int, width: int, height: int, max_depth=8,
+                       flags=0, block=0) -> Workload:
+    w = Workload(kind=WL_PATHTRACE, flags=flags, block_threads=block)
+    w.pathtrace = PathtraceParams(scene_ptr, scene_bytes, width, height, max_depth)
     return w
 
 
