@@ -404,6 +404,24 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
                      "fma_frac_of_peak": c.n_threads * c.fma_count / (t * 1e-3) / fma_peak}
     res["speedup_vs_pdom"] = res["spec_call"]["value"] / res["pdom"]["value"]
     out["commoncall"] = res
+
+    # configs[3]: path tracer, 1024^2 x 16 spp over the 1,044,494-triangle BVH scene
+    c = I.C4
+    tris, mat, mats, cam = I.cornell_scene(c)
+    buf, used = sr.upload_scene(tris, mat, mats, cam, ctx.device)
+    w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth)
+    ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
+    res = {"scene_triangles": int(len(tris)), "scene_bytes": int(used)}
+    for name, mode, thr in (("pdom", sr.PDOM, 0), ("spec_t32", sr.SPEC_LOOP, 32)):
+        ms = timer.time_steps(lambda: sr.sr_run(w, c.n_pixels, c.spp, I.PRIMARY_SEED, mode, thr),
+                              max(3, min(args.steps, 5)), 1)
+        t = statistics.median(ms)
+        cnt = ctx.region(w, c.n_pixels, sr.T_COUNTERS, torch.int64).cpu().numpy()
+        res[name] = {"value": c.n_pixels * c.spp / (t * 1e-3), "unit": "paths/s", "ms": t,
+                     "rays": int(cnt[1]), "node_visits": int(cnt[2]), "tri_tests": int(cnt[3]),
+                     "launch": sr.sr_last_launch()}
+    res["speedup_vs_pdom"] = res["spec_t32"]["value"] / res["pdom"]["value"]
+    out["pathtrace"] = res
     return out
 
 

@@ -14,7 +14,7 @@ from paper_conf_cgo_damanijskymg20_b200 import inputs as I  # noqa: E402
 from paper_conf_cgo_damanijskymg20_b200 import sr  # noqa: E402
 
 ap = argparse.ArgumentParser()
-ap.add_argument("what", nargs="*", default=["divloop", "commoncall", "mcml"])
+ap.add_argument("what", nargs="*", default=["divloop", "commoncall", "mcml", "pathtrace"])
 ap.add_argument("--photons", type=int, default=I.C3.n_photons)
 ap.add_argument("--modes", default="pdom,spec")
 ap.add_argument("--threshold", type=int, default=32)
@@ -44,6 +44,16 @@ if "mcml" in a.what:
     ctx.ensure(sr.sr_workspace_bytes(w, nt))
     for md in modes:
         sr.sr_run(w, nt, m.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
+                  0 if md == "pdom" else a.threshold)
+if "pathtrace" in a.what:
+    c = I.C4
+    tris, mat, mats, cam = I.cornell_scene(c)
+    buf, used = sr.upload_scene(tris, mat, mats, cam)
+    w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth,
+                              flags=sr.F_STATIC)
+    ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
+    for md in modes:
+        sr.sr_run(w, c.n_pixels, c.spp, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
                   0 if md == "pdom" else a.threshold)
 torch.cuda.synchronize()
 sr.sr_finalize()

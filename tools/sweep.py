@@ -93,5 +93,21 @@ if "divloop" in a.what:
             res.append(r)
             print(json.dumps(r), file=sys.stderr, flush=True)
     out["divloop"] = res
+if "pathtrace" in a.what:
+    c = I.C4
+    tris, mat, mats, cam = I.cornell_scene(c)
+    buf, used = sr.upload_scene(tris, mat, mats, cam)
+    res = []
+    for b in blocks:
+        w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth, block=b)
+        ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
+        for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
+            t = timed(lambda: sr.sr_run(w, c.n_pixels, c.spp, seed, mode, T), a.reps)
+            r = dict(block=b, mode="pdom" if mode == sr.PDOM else "spec", T=T, ms=t,
+                     paths_per_s=c.n_pixels * c.spp / (t * 1e-3), launch=sr.sr_last_launch())
+            r.update(eff(w, c.n_pixels, c.spp, mode, T))
+            res.append(r)
+            print(json.dumps(r), file=sys.stderr, flush=True)
+    out["pathtrace"] = res
 print(json.dumps(out))
 sr.sr_finalize()
