@@ -64,6 +64,9 @@ typedef enum {
 #define SR_F_STATIC 2u  /* MCML / PATHTRACE: static task->lane assignment (lane l owns tasks
                            l + k*n_threads) instead of the default dynamic per-warp claiming.
                            Results are identical; only the schedule differs. */
+#define SR_F_COARSE 4u  /* PATHTRACE + SR_SPEC_LOOP: merge at bounce granularity (one release =
+                           traversal + shading of one bounce) instead of the default BVH-node
+                           granularity (one release = one node visit). Results are identical. */
 
 #define SR_MAX_LAYERS 8
 typedef struct { float n, mua, mus, g, d; } sr_layer;  /* -, 1/cm, 1/cm, -, cm */

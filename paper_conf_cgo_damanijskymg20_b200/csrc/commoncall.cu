@@ -44,29 +44,29 @@ __device__ __forceinline__ void count_call(uint32_t& execs, uint32_t& lanes) {
 
 template <int ROUNDS, bool SCHED>
 __global__ void __launch_bounds__(1024) commoncall_pdom(const CallArgs a) {
-  const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
   if (g >= a.n) return;
   const uint64_t t = a.t0 + g;
   float ysum = 0.0f;
   uint32_t then_cnt = 0, execs = 0, lanes = 0;
-  for (uint32_t it = 0; it < a.iters; ++it) {
+  for (uint32_t it = 0; it < a.iters; ++it) {  // @sr-region MERGE:full
     const uint4 u = draw(it, kTagCall, t, a.seed);
     const float x = u01(u.y);
     float y;
     if (u.x < a.split_u32) {                 // then-arm
-      count_call<SCHED>(execs, lanes);
+      count_call<SCHED>(execs, lanes);  // @sr-region THEN
       y = foo<ROUNDS>(x, a.rounds);          // call site 1
       ++then_cnt;
     } else {                                 // else-arm
-      float x1 = x * 0.5f;
+      float x1 = x * 0.5f;  // @sr-region ELSE_PRE
       x1 = x1 + 0.25f;
       count_call<SCHED>(execs, lanes);
-      y = foo<ROUNDS>(x1, a.rounds);         // call site 2
-      y = y * y;
-    }                                        // IPDOM: original reconvergence point
+      y = foo<ROUNDS>(x1, a.rounds);         // call site 2 (still ELSE_PRE's mask)
+      y = y * y;  // @sr-region ELSE_POST
+    }  // @sr-region MERGE:full
     ysum = ysum + y;
   }
-  a.y[g] = ysum;
+  a.y[g] = ysum;  // @sr-region ENTRY:full
   const uint32_t vm = valid_mask(g & ~31ull, a.n);
   const uint32_t tot = __reduce_add_sync(vm, then_cnt);
   uint32_t e = 0, l = 0;
@@ -79,17 +79,17 @@ __global__ void __launch_bounds__(1024) commoncall_pdom(const CallArgs a) {
       p[1] = make_uint4(0u, 0u, 0u, 0u);
     }
   }
-}
+}  // @sr-region END
 
 template <int ROUNDS, bool SCHED>
 __global__ void __launch_bounds__(1024) commoncall_spec(const CallArgs a) {
-  const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
   if (g >= a.n) return;
   const uint32_t vm = valid_mask(g & ~31ull, a.n);
   const uint64_t t = a.t0 + g;
   float ysum = 0.0f;
   uint32_t then_cnt = 0, execs = 0, lanes = 0;
-  for (uint32_t it = 0; it < a.iters; ++it) {
+  for (uint32_t it = 0; it < a.iters; ++it) {  // @sr-region MERGE:full
     const uint4 u = draw(it, kTagCall, t, a.seed);
     const float x = u01(u.y);
     const bool c = u.x < a.split_u32;
@@ -98,14 +98,14 @@ __global__ void __launch_bounds__(1024) commoncall_spec(const CallArgs a) {
       arg = x * 0.5f;
       arg = arg + 0.25f;
     }
-    __syncwarp(vm);                          // reconverge at foo's entry
+    __syncwarp(vm);  // @sr-region CALL
     count_call<SCHED>(execs, lanes);
     float y = foo<ROUNDS>(arg, a.rounds);    // the one call, all lanes
-    if (!c) y = y * y;                       // else-arm suffix
+    if (!c) y = y * y;  // @sr-region MERGE:full
     ysum = ysum + y;
     then_cnt += c ? 1u : 0u;
   }
-  a.y[g] = ysum;
+  a.y[g] = ysum;  // @sr-region ENTRY:full
   const uint32_t tot = __reduce_add_sync(vm, then_cnt);
   uint32_t e = 0, l = 0;
   if constexpr (SCHED) { e = __reduce_add_sync(vm, execs); l = __reduce_add_sync(vm, lanes); }
@@ -117,7 +117,7 @@ __global__ void __launch_bounds__(1024) commoncall_spec(const CallArgs a) {
       p[1] = make_uint4(0u, 0u, 0u, 0u);
     }
   }
-}
+}  // @sr-region END
 
 template <bool SCHED>
 cudaError_t launch_t(const LaunchCtx& c, const CallArgs& a, int mode) {

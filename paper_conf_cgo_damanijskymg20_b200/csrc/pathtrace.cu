@@ -109,60 +109,80 @@ __device__ __forceinline__ void tri_test(const PtTri& T, V3 o, V3 d, float& tb, 
   }
 }
 
-__device__ int64_t closest_hit(const PtArgs& a, V3 o, V3 d, float& t_out, uint32_t& mat_out,
-                               uint32_t& tri_slot, Stats& st) {
-  const V3 inv = mk(1.0f / d.x, 1.0f / d.y, 1.0f / d.z);
-  float tb = INFINITY;
-  int64_t ib = -1;
-  uint32_t mb = 0;
+// Resumable BVH traversal: one call of trav_step visits one node (its two
+// child boxes, the triangles of child leaves, push/pop).  closest_hit() runs
+// it to completion; the node-granularity Loop Merge kernel interleaves single
+// steps of different lanes' rays.
+struct Trav {
+  V3 o, d, inv;
+  float tb;
+  int64_t ib;
+  uint32_t mb, slot;
+  int32_t node;
+  int32_t sp;
   int32_t stack[kStack];
-  int sp = 0;
-  int32_t node = 0;
-  uint32_t slot = 0;
-  for (;;) {
-    const PtNode N = a.nodes[node];
-    ++st.nodes;
-    float tn0, tn1;
-    const bool h0 = N.cnt0 >= 0 && N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, inv, tb, tn0);
-    const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, o, inv, tb, tn1);
-    int32_t next = -1;
-    // leaves: test their triangles now; inner children: descend / push
-    if (h0 && N.cnt0 > 0) {
-      for (int32_t k = 0; k < N.cnt0; ++k) {
-        const int64_t before = ib;
-        tri_test(a.tris[N.ref0 + k], o, d, tb, ib, mb);
-        if (ib != before) slot = (uint32_t)(N.ref0 + k);
-        ++st.tests;
-      }
+};
+
+__device__ __forceinline__ void trav_begin(Trav& tr, V3 o, V3 d) {
+  tr.o = o;
+  tr.d = d;
+  tr.inv = mk(1.0f / d.x, 1.0f / d.y, 1.0f / d.z);
+  tr.tb = INFINITY;
+  tr.ib = -1;
+  tr.mb = 0;
+  tr.slot = 0;
+  tr.node = 0;
+  tr.sp = 0;
+}
+
+// returns false when the traversal is finished
+__device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) {
+  const PtNode N = a.nodes[tr.node];
+  ++st.nodes;
+  float tn0, tn1;
+  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, tr.o, tr.inv, tr.tb, tn0);
+  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, tr.o, tr.inv, tr.tb, tn1);
+  // leaves: test their triangles now; inner children: descend / push
+  if (h0 && N.cnt0 > 0) {
+    for (int32_t k = 0; k < N.cnt0; ++k) {
+      const int64_t before = tr.ib;
+      tri_test(a.tris[N.ref0 + k], tr.o, tr.d, tr.tb, tr.ib, tr.mb);
+      if (tr.ib != before) tr.slot = (uint32_t)(N.ref0 + k);
+      ++st.tests;
     }
-    if (h1 && N.cnt1 > 0) {
-      for (int32_t k = 0; k < N.cnt1; ++k) {
-        const int64_t before = ib;
-        tri_test(a.tris[N.ref1 + k], o, d, tb, ib, mb);
-        if (ib != before) slot = (uint32_t)(N.ref1 + k);
-        ++st.tests;
-      }
-    }
-    const bool in0 = h0 && N.cnt0 == 0, in1 = h1 && N.cnt1 == 0;
-    if (in0 && in1) {
-      const bool first0 = tn0 <= tn1;
-      next = first0 ? N.ref0 : N.ref1;
-      if (sp < kStack) stack[sp++] = first0 ? N.ref1 : N.ref0;
-    } else if (in0) {
-      next = N.ref0;
-    } else if (in1) {
-      next = N.ref1;
-    }
-    if (next < 0) {
-      if (sp == 0) break;
-      next = stack[--sp];
-    }
-    node = next;
   }
-  t_out = tb;
-  mat_out = mb;
-  tri_slot = slot;
-  return ib;
+  if (h1 && N.cnt1 > 0) {
+    for (int32_t k = 0; k < N.cnt1; ++k) {
+      const int64_t before = tr.ib;
+      tri_test(a.tris[N.ref1 + k], tr.o, tr.d, tr.tb, tr.ib, tr.mb);
+      if (tr.ib != before) tr.slot = (uint32_t)(N.ref1 + k);
+      ++st.tests;
+    }
+  }
+  const bool in0 = h0 && N.cnt0 == 0, in1 = h1 && N.cnt1 == 0;
+  int32_t next = -1;
+  if (in0 && in1) {
+    const bool first0 = tn0 <= tn1;
+    next = first0 ? N.ref0 : N.ref1;
+    if (tr.sp < kStack) tr.stack[tr.sp++] = first0 ? N.ref1 : N.ref0;
+  } else if (in0) {
+    next = N.ref0;
+  } else if (in1) {
+    next = N.ref1;
+  }
+  if (next < 0) {
+    if (tr.sp == 0) return false;
+    next = tr.stack[--tr.sp];
+  }
+  tr.node = next;
+  return true;
+}
+
+__device__ __forceinline__ int64_t closest_hit(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
+  trav_begin(tr, o, d);
+  while (trav_step(a, tr, st)) {
+  }
+  return tr.ib;
 }
 
 struct Path {
@@ -199,14 +219,14 @@ __device__ __forceinline__ void onb(V3 n, V3& t1, V3& t2) {
   t2 = mk(b, sign + n.y * n.y * a, -n.y);
 }
 
-// One bounce (the common inner-loop body).  Ends the path when it escapes,
-// hits a light, reaches max_depth or loses the roulette; the epilog (pixel
-// sum) happens at that point, in sample order.
-__device__ void bounce(const PtArgs& a, Path& p, Stats& st) {
-  float t;
-  uint32_t mat, slot;
-  const int64_t hit = closest_hit(a, p.o, p.d, t, mat, slot, st);
-  ++st.rays;
+// The shading half of a bounce, after the closest hit of ray (p.o, p.d) is
+// known (tr finished).  Ends the path when it escaped, hit a light, reached
+// max_depth or lost the roulette; the epilog (pixel sum) happens at that
+// point, in sample order.
+__device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
+  const int64_t hit = tr.ib;
+  const float t = tr.tb;
+  const uint32_t mat = tr.mb, slot = tr.slot;
   bool end = hit < 0;
   if (!end) {
     const PtMat m = a.mats[mat];
@@ -292,6 +312,12 @@ __device__ __forceinline__ void finish(const PtArgs& a, const Path& p, bool vali
   }
 }
 
+__device__ __forceinline__ void bounce(const PtArgs& a, Path& p, Trav& tr, Stats& st) {
+  closest_hit(a, tr, p.o, p.d, st);
+  ++st.rays;
+  shade(a, p, tr);
+}
+
 template <bool SCHED>
 __global__ void __launch_bounds__(128) pt_pdom(const PtArgs a) {
   const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
@@ -301,6 +327,7 @@ __global__ void __launch_bounds__(128) pt_pdom(const PtArgs a) {
   p.pix = (uint32_t)(valid ? g : 0);
   p.sum = mk(0.0f, 0.0f, 0.0f);
   p.alive = false;
+  Trav tr;
   Stats st{0, 0, 0};
   uint32_t paths = 0, outer = 0, rel = 0, rel_lanes = 0, launch_lanes = 0;
   for (uint32_t s = 0; s < a.spp; ++s) {
@@ -314,7 +341,7 @@ __global__ void __launch_bounds__(128) pt_pdom(const PtArgs a) {
           const uint32_t m = __activemask();
           if (lane_id() == (uint32_t)(__ffs(m) - 1)) { ++rel; rel_lanes += __popc(m); }
         }
-        bounce(a, p, st);
+        bounce(a, p, tr, st);
       } while (p.alive);
     }                                   // IPDOM: reconverge, next sample
   }
@@ -323,7 +350,14 @@ __global__ void __launch_bounds__(128) pt_pdom(const PtArgs a) {
   finish(a, p, valid, st, paths, g >> 5, outer, r, rl, outer, launch_lanes);
 }
 
-template <bool SCHED>
+// Loop Merge.  NODE = false: the merged inner loop is the bounce loop (one
+// release = one whole bounce: traversal + shading).  NODE = true: the merged
+// inner loop is the BVH traversal itself (one release = one node visit for
+// every lane with a ray in flight); shading, the pixel epilog and the next
+// camera ray form the advance step.  The second is Loop Merge applied one
+// nesting level deeper (P:1514-1528 leaves nesting open), where the trip
+// count (nodes per ray) varies most.
+template <bool SCHED, bool NODE>
 __global__ void __launch_bounds__(128) pt_spec(const PtArgs a) {
   const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -333,29 +367,40 @@ __global__ void __launch_bounds__(128) pt_spec(const PtArgs a) {
   p.sum = mk(0.0f, 0.0f, 0.0f);
   p.alive = false;
   p.s = 0;
+  Trav tr;
+  bool trav = false;                   // NODE: a ray of this lane is being traversed
   Stats st{0, 0, 0};
   uint32_t paths = 0, rounds = 0, rel = 0, rel_lanes = 0, adv = 0, adv_lanes = 0;
   uint32_t next_s = 0;
-  uint32_t E = __ballot_sync(kFull, !valid || a.spp == 0);  // lanes with no sample left
+  uint32_t E = __ballot_sync(kFull, !valid || a.spp == 0);  // lanes with nothing left to do
   for (;;) {
-    const uint32_t P = __ballot_sync(kFull, p.alive);
+    const uint32_t P = __ballot_sync(kFull, NODE ? trav : p.alive);
     const uint32_t R = ~(P | E);
     if ((P | R) == 0u) break;
     if constexpr (SCHED) ++rounds;
     if ((uint32_t)__popc(P) >= a.T || R == 0u) {
       if constexpr (SCHED) { ++rel; rel_lanes += __popc(P); }
-      if (p.alive) {
+      if ((P >> lane_id()) & 1u) {
         __syncwarp(P);
-        bounce(a, p, st);
+        if constexpr (NODE) trav = trav_step(a, tr, st);
+        else bounce(a, p, tr, st);
       }
     } else {
       if constexpr (SCHED) { ++adv; adv_lanes += __popc(R); }
       if ((R >> lane_id()) & 1u) {
-        p.s = next_s++;
-        camera_ray(a, H, p);
-        ++paths;
+        if (NODE && p.alive) shade(a, p, tr);        // finish the bounce whose ray is done
+        if (!p.alive && next_s < a.spp) {             // epilog done in shade; next sample
+          p.s = next_s++;
+          camera_ray(a, H, p);
+          ++paths;
+        }
+        if (NODE && p.alive) {                        // start the next ray
+          trav_begin(tr, p.o, p.d);
+          ++st.rays;
+          trav = true;
+        }
       }
-      E = __ballot_sync(kFull, !valid || next_s >= a.spp);  // no sample left to start
+      E = __ballot_sync(kFull, !valid || (!p.alive && next_s >= a.spp));
     }
   }
   finish(a, p, valid, st, paths, g >> 5, rounds, rel, rel_lanes, adv, adv_lanes);
@@ -367,11 +412,10 @@ __global__ void pt_query(const PtArgs a) {
   if (i >= a.n) return;
   const float* r = a.q_rays + 6 * i;
   Stats st{0, 0, 0};
-  float t;
-  uint32_t mat, slot;
-  const int64_t h = closest_hit(a, mk(r[0], r[1], r[2]), mk(r[3], r[4], r[5]), t, mat, slot, st);
+  Trav tr;
+  const int64_t h = closest_hit(a, tr, mk(r[0], r[1], r[2]), mk(r[3], r[4], r[5]), st);
   a.q_hit[i] = h;
-  a.q_t[i] = t;
+  a.q_t[i] = tr.tb;
 }
 
 PtArgs base_args(const void* scene) {
@@ -429,12 +473,17 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
   if (grid > 0x7fffffffull) return cudaErrorInvalidConfiguration;
   record_launch((uint32_t)grid, block, 0);
   const bool spec = mode == SR_SPEC_LOOP;
-  if (a.sched) {
-    if (spec) pt_spec<true><<<(unsigned)grid, block, 0, c.stream>>>(a);
-    else pt_pdom<true><<<(unsigned)grid, block, 0, c.stream>>>(a);
+  const bool node = (w.flags & SR_F_COARSE) == 0;
+  const unsigned gr = (unsigned)grid;
+  if (!spec) {
+    if (a.sched) pt_pdom<true><<<gr, block, 0, c.stream>>>(a);
+    else pt_pdom<false><<<gr, block, 0, c.stream>>>(a);
+  } else if (node) {
+    if (a.sched) pt_spec<true, true><<<gr, block, 0, c.stream>>>(a);
+    else pt_spec<false, true><<<gr, block, 0, c.stream>>>(a);
   } else {
-    if (spec) pt_spec<false><<<(unsigned)grid, block, 0, c.stream>>>(a);
-    else pt_pdom<false><<<(unsigned)grid, block, 0, c.stream>>>(a);
+    if (a.sched) pt_spec<true, false><<<gr, block, 0, c.stream>>>(a);
+    else pt_spec<false, false><<<gr, block, 0, c.stream>>>(a);
   }
   return cudaGetLastError();
 }

@@ -78,12 +78,13 @@ def render(ctx, cfg, mode, T, flags=0, block=0):
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 8),
                                     (sr.SPEC_LOOP, 32)])
 @pytest.mark.parametrize("block", [32, 128])
-def test_render_bit_exact_small(ctx, mode, T, block):
+@pytest.mark.parametrize("flags", [0, sr.F_COARSE])
+def test_render_bit_exact_small(ctx, mode, T, block, flags):
     cfg = I.C4_SMALL
     tris, mat, mats, cam, buf, used = scene(cfg)
     ref, rc = oracle.pt_render(oracle.pt_scene(tris, mat, mats, cam), cfg.width, cfg.height,
                                cfg.spp, cfg.max_depth, I.PRIMARY_SEED)
-    rgb, cnt = render(ctx, cfg, mode, T, block=block)
+    rgb, cnt = render(ctx, cfg, mode, T, block=block, flags=flags)
     assert np.array_equal(rgb.view(np.uint32), ref.view(np.uint32))
     assert cnt[0] == rc["paths"] and cnt[1] == rc["rays"]
 
@@ -92,8 +93,10 @@ def test_render_full_config_invariants_and_sampled_pixels(ctx):
     cfg = I.C4
     a, ca = render(ctx, cfg, sr.SPEC_LOOP, 32)
     b, cb = render(ctx, cfg, sr.PDOM, 0)
+    c, cc = render(ctx, cfg, sr.SPEC_LOOP, 16, flags=sr.F_COARSE)
     assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
-    assert np.array_equal(ca, cb)
+    assert np.array_equal(a.view(np.uint32), c.view(np.uint32))
+    assert np.array_equal(ca, cb) and np.array_equal(ca, cc)
     assert ca[0] == cfg.n_pixels * cfg.spp
     tris, mat, mats, cam, buf, used = scene(cfg)
     pix = np.array([0, 1023, 512 * 1024 + 512, 700 * 1024 + 300, 1024 * 1024 - 1, 123457],

@@ -1,0 +1,200 @@
+"""Static per-region SASS instruction counts of the built kernels (no GPU).
+
+The warp simulator (oracle/warpsim.c) counts, per source region of the hot
+path, warp executions and active lanes.  SIMT efficiency needs the
+cost of each region in SASS instructions; this tool reads it off the cubin in
+libsr.so:
+
+  * regions are delimited in the CUDA source by `// @sr-region NAME[:full]`
+    comments (a marker applies from its line to the next marker);
+  * every SASS instruction is attributed to the innermost frame of its inline
+    chain (nvdisasm -gi) that lies in a marked region (so a marked device
+    function such as the MC step splits into its own regions, while unmarked
+    helpers such as Philox count toward their call site);
+  * cold code is excluded: the slow path of BRA.DIV (WARPSYNC.COLLECTIVE
+    sequences), the trailing self-branch/NOP padding, and subroutines reached
+    by CALL.REL (IEEE div/sqrt slow paths);
+  * a CALL.ABS to a non-inlined device function (foo of config 2) adds the
+    callee's instruction count to the calling region.
+
+`:full` marks code executed by every valid lane of the warp whenever the
+region's scheduler step runs (round bookkeeping, branch headers), as opposed
+to the lanes the simulator puts in that region's mask.
+
+usage: python tools/sass_regions.py [kernel-regex]   -> JSON on stdout
+"""
+from __future__ import annotations
+
+import json
+import os
+import re
+import subprocess
+import sys
+import tempfile
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+LIB = os.path.join(ROOT, "paper_conf_cgo_damanijskymg20_b200", "libsr.so")
+CSRC = os.path.join(ROOT, "paper_conf_cgo_damanijskymg20_b200", "csrc")
+
+LINE_RE = re.compile(r'//## File "([^"]+)", line (\d+)(.*)')
+INL_RE = re.compile(r'inlined at "([^"]+)", line (\d+)')
+INS_RE = re.compile(r"/\*([0-9a-f]{4,})\*/\s+(.*?)\s*;")
+MARK_RE = re.compile(r"//\s*@sr-region\s+([A-Z_0-9]+)(:full)?")
+
+
+def region_map(path):
+    """line -> (region, full) from the @sr-region markers of one source file."""
+    out, cur = {}, None
+    for i, line in enumerate(open(path), 1):
+        m = MARK_RE.search(line)
+        if m:
+            cur = None if m.group(1) == "END" else (m.group(1), bool(m.group(2)))
+        if cur is not None:
+            out[i] = cur
+    return out
+
+
+def extract_cubins(tmp):
+    subprocess.run(["cuobjdump", "-xelf", "all", LIB], cwd=tmp, capture_output=True)
+    return [os.path.join(tmp, f) for f in os.listdir(tmp) if f.endswith(".cubin")]
+
+
+def parse_functions(cubin):
+    """{function: [dict(addr, text, file, line, outer_file, outer_line, label_before)]}"""
+    txt = subprocess.run(["nvdisasm", "-gi", "-c", cubin], capture_output=True, text=True).stdout
+    funcs, cur, loc, labels = {}, None, (None, None, None, None, []), []
+    for raw in txt.splitlines():
+        m = re.match(r"\s*\.text\.(\S+):", raw)
+        if m:
+            cur = m.group(1)
+            funcs[cur] = []
+            continue
+        if cur is None:
+            continue
+        m = LINE_RE.search(raw)
+        if m:
+            f, ln, rest = m.group(1), int(m.group(2)), m.group(3)
+            inl = INL_RE.findall(rest)
+            of, ol = (inl[-1][0], int(inl[-1][1])) if inl else (f, ln)
+            chain = [(f, ln)] + [(a, int(b)) for a, b in inl]   # innermost -> outermost
+            loc = (f, ln, of, ol, chain)
+            continue
+        m = re.match(r"^(\.L_x_\d+|\$\S+):$", raw.strip())
+        if m:
+            labels.append(m.group(1))
+            continue
+        m = INS_RE.search(raw)
+        if m:
+            funcs[cur].append(dict(addr=int(m.group(1), 16), text=m.group(2), file=loc[0],
+                                   line=loc[1], outer_file=loc[2], outer_line=loc[3],
+                                   chain=loc[4], labels=labels))
+            labels = []
+    return funcs
+
+
+def cold_set(ins):
+    """Indices of instructions on cold paths."""
+    label_at = {}
+    for i, x in enumerate(ins):
+        for lb in x["labels"]:
+            label_at[lb] = i
+    cold = set()
+    # 1. BRA.DIV slow paths and CALL.REL subroutines: from the target label up
+    #    to (and including) the block's terminating branch back / RET
+    starts = []
+    for x in ins:
+        m = re.search(r"BRA\.DIV\s+\S+,\s*`\((\.L_x_\d+)\)", x["text"])
+        if m:
+            starts.append(m.group(1))
+    for lb in starts:
+        i = label_at.get(lb)
+        while i is not None and i < len(ins):
+            cold.add(i)
+            t = ins[i]["text"]
+            if re.match(r"(@\S+\s+)?(RET|BRA)\b", t) and not t.startswith("@"):
+                break
+            i += 1
+    # 2. trailing trap loop / padding
+    for i, x in enumerate(ins):
+        m = re.search(r"BRA\s+`\((\.L_x_\d+)\)", x["text"])
+        if m and label_at.get(m.group(1)) == i:
+            cold.update(range(i, len(ins)))
+            break
+    return cold
+
+
+def loop_intervals(ins):
+    """[start, end] index ranges of loops (a branch back to an earlier label)."""
+    label_at = {}
+    for i, x in enumerate(ins):
+        for lb in x["labels"]:
+            label_at[lb] = i
+    out = []
+    for i, x in enumerate(ins):
+        m = re.search(r"\bBRA\b.*`\((\.L_x_\d+)\)", x["text"])
+        if m and "BRA.DIV" not in x["text"]:
+            j = label_at.get(m.group(1))
+            if j is not None and j < i:
+                out.append((j, i))
+    return out
+
+
+def kernel_costs(kernel_regex=".*"):
+    maps = {}
+    for f in os.listdir(CSRC):
+        if f.endswith(".cu"):
+            maps[os.path.join(CSRC, f)] = region_map(os.path.join(CSRC, f))
+    with tempfile.TemporaryDirectory() as tmp:
+        funcs = {}
+        for c in extract_cubins(tmp):
+            funcs.update(parse_functions(c))
+    out = {}
+    for name, ins in funcs.items():
+        if not re.search(kernel_regex, name) or "foo" in name:
+            continue
+        # split the section: kernel body, then subroutines ($kernel$callee labels)
+        subs, body_end = {}, len(ins)
+        cur = None
+        for i, x in enumerate(ins):
+            for lb in x["labels"]:
+                if lb.startswith("$"):
+                    cur = lb
+                    body_end = min(body_end, i)
+                    subs[cur] = []
+            if cur is not None:
+                subs[cur].append(x)
+        body = ins[:body_end]
+        sub_size = {}
+        for lb, si in subs.items():
+            hot = "__internal" not in lb   # IEEE div/sqrt slow paths are cold
+            sub_size[lb] = len(si) if hot else 0
+        cold = cold_set(body)
+        loops = [(a, b) for a, b in loop_intervals(body) if a not in cold and b not in cold]
+        reg = {}
+        unmapped = 0
+        for i, x in enumerate(body):
+            if i in cold:
+                continue
+            # the innermost inline frame that lies in a marked region decides
+            r = None
+            for f, ln in x["chain"]:
+                r = maps.get(f, {}).get(ln)
+                if r is not None:
+                    break
+            if r is None:
+                unmapped += 1
+                r = ("UNMAPPED", True)
+            if r[0] != "ENTRY" and loops and not any(a <= i <= b for a, b in loops):
+                r = ("ENTRY", True)   # loop preheader / exit copy: runs once per warp
+            key = r[0] + (":full" if r[1] else "")
+            n = 1
+            cm = re.search(r"CALL\.\w+(?:\.NOINC)?\s+`\((\S+?)\)", x["text"])
+            if cm and cm.group(1) in sub_size and not x["text"].startswith("@"):
+                n += sub_size[cm.group(1)]
+            reg[key] = reg.get(key, 0) + n
+        out[name] = dict(regions=reg, unmapped=unmapped, total=sum(reg.values()))
+    return out
+
+
+if __name__ == "__main__":
+    print(json.dumps(kernel_costs(sys.argv[1] if len(sys.argv) > 1 else ".*"), indent=1))

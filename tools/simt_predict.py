@@ -1,0 +1,103 @@
+"""Predict whole-kernel SIMT efficiency with the warp simulator (oracle part
+2) and the static SASS region costs of the built cubin (tools/sass_regions.py),
+and compare with the ncu measurement in profiles/simt_efficiency.json.
+
+SIMT efficiency = thread-instructions / (32 x warp-instructions);
+predicted = sum_r c_r L_r / (32 sum_r c_r X_r), where for each SASS region r
+with cost c_r the simulator supplies X_r warp executions and L_r active lanes
+over every warp of the launch ("X:full" regions run with every valid lane
+whenever step X runs; ENTRY once per warp).
+
+TEST/EVALUATION INFRASTRUCTURE: uses oracle/ (event streams + simulator).
+
+usage: python tools/simt_predict.py  -> JSON (and profiles/simt_prediction.json with --write)
+"""
+from __future__ import annotations
+
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tools"))
+
+import numpy as np  # noqa: E402
+
+import oracle  # noqa: E402
+import sass_regions  # noqa: E402
+from paper_conf_cgo_damanijskymg20_b200 import inputs as I  # noqa: E402
+
+
+def accumulate(costs, sim, n_valid, acc):
+    for key, c in costs.items():
+        name, full = key.split(":")[0], key.endswith(":full")
+        if name in ("ENTRY", "UNMAPPED"):
+            x, l = 1, n_valid
+        else:
+            x, ln = sim[name]
+            l = x * n_valid if full else ln
+        acc[0] += c * x
+        acc[1] += c * l
+
+
+def predict(costs, warps):
+    """warps: iterable of (sim_counts_dict, n_valid)."""
+    acc = [0, 0]
+    for sim, nv in warps:
+        accumulate(costs, sim, nv, acc)
+    return dict(inst=acc[0], thread_inst=acc[1], simt=acc[1] / (32.0 * acc[0]))
+
+
+def find(costs_all, pattern):
+    import re
+    for k, v in costs_all.items():
+        if re.search(pattern, k):
+            return v["regions"]
+    raise KeyError(pattern)
+
+
+def divloop_warps(mode, T):
+    c = I.C1
+    want = oracle.divloop_wants(0, c.n_threads, c.iters, I.PRIMARY_SEED, c.p_u32)
+    for w in range(0, c.n_threads, 32):
+        ww = want[w:w + 32]
+        yield oracle.ws_divloop(ww, mode, T), len(ww)
+
+
+def commoncall_warps(mode):
+    c = I.C2
+    _, arm = oracle.commoncall(0, c.n_threads, 1, I.PRIMARY_SEED, c.split_u32, fma_count=0)
+    for w in range(0, c.n_threads, 32):
+        a = arm[w:w + 32]
+        yield oracle.ws_commoncall(a, mode), len(a)
+
+
+def main():
+    costs = sass_regions.kernel_costs("divloop_|commoncall_")
+    measured = json.load(open(os.path.join(ROOT, "profiles", "simt_efficiency.json")))
+    rows = {}
+    cases = [
+        ("divloop_pdom", r"divloop_pdomILi125ELb0", lambda: divloop_warps(oracle.PDOM, 0)),
+        ("divloop_spec(T=16)", r"divloop_specILi125ELb0", lambda: divloop_warps(oracle.SPEC_LOOP, 16)),
+        ("commoncall_pdom", r"commoncall_pdomILi250ELb0", lambda: commoncall_warps(oracle.PDOM)),
+        ("commoncall_spec", r"commoncall_specILi250ELb0", lambda: commoncall_warps(oracle.SPEC_CALL)),
+    ]
+    for label, pat, gen in cases:
+        p = predict(find(costs, pat), gen())
+        m = measured.get(label, {})
+        rows[label] = dict(predicted=p["simt"], measured=m.get("simt_efficiency"),
+                           predicted_inst=p["inst"], measured_inst=m.get("inst"),
+                           predicted_thread_inst=p["thread_inst"],
+                           measured_thread_inst=m.get("thread_inst"),
+                           costs=find(costs, pat))
+        if m.get("simt_efficiency") is not None:
+            rows[label]["abs_err_points"] = 100 * abs(p["simt"] - m["simt_efficiency"])
+    out = json.dumps(rows, indent=1)
+    if "--write" in sys.argv:
+        open(os.path.join(ROOT, "profiles", "simt_prediction.json"), "w").write(out + "\n")
+    print(out)
+
+
+if __name__ == "__main__":
+    main()
