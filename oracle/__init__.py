@@ -30,7 +30,10 @@ PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
 DL = dict(ENTRY=0, PROLOG=1, EXPENSIVE=2, EPILOG=3, ROUND=4, RELEASE=5, ADVANCE=6)
 CC = dict(ENTRY=0, THEN=1, ELSE_PRE=2, CALL=3, ELSE_POST=4, MERGE=5)
 LM = dict(ENTRY=0, LAUNCH=1, STEP=2, STEP_BOUNDARY=3, STEP_INTERACT=4, ROUND=5, RELEASE=6,
-          ADVANCE=7)
+          ADVANCE=7, **{f"EV{b}": 8 + b for b in range(8)}, **{f"NEV{b}": 16 + b for b in range(8)})
+# MC step event bits (oracle.h OR_EV_*)
+EV_BOUNDARY, EV_SLEFT, EV_REFLECT, EV_EXIT, EV_TRANSMIT, EV_ROULETTE, EV_SPIN_AXIS, \
+    EV_SPIN_GENERAL = 1, 2, 4, 8, 16, 32, 64, 128
 MC_COUNTERS = ["photons", "steps", "rd_exits", "tt_exits", "rr_kills", "rr_survive", "capped",
                "zero_w"]
 MAX_LAYERS = 8
@@ -58,7 +61,7 @@ class MCParams(C.Structure):
 
 
 class WsCounts(C.Structure):
-    _fields_ = [("rounds", C.c_uint64), ("execs", C.c_uint64 * 16), ("lanes", C.c_uint64 * 16)]
+    _fields_ = [("rounds", C.c_uint64), ("execs", C.c_uint64 * 24), ("lanes", C.c_uint64 * 24)]
 
     def as_dict(self, names):
         return {"rounds": int(self.rounds),
@@ -192,6 +195,24 @@ def mcml_events(p: MCParams, pid, seed, cap=1 << 20):
     return ev[:n].copy()
 
 
+def mcml_events_batch(p: MCParams, id0, count, seed, cap=None):
+    """(ev uint8[total], off uint64[count], nsteps uint32[count])"""
+    L = lib()
+    L.or_mcml_events_batch.argtypes = [C.POINTER(MCParams), C.c_uint64, C.c_uint64, C.c_uint64,
+                                       C.POINTER(C.c_uint8), C.c_uint64,
+                                       C.POINTER(C.c_uint64), C.POINTER(C.c_uint32)]
+    L.or_mcml_events_batch.restype = C.c_uint64
+    cap = cap or count * 2000
+    ev = np.zeros(cap, np.uint8)
+    off = np.zeros(count, np.uint64)
+    ns = np.zeros(count, np.uint32)
+    used = L.or_mcml_events_batch(C.byref(p), id0, count, seed, _p(ev, C.c_uint8), cap,
+                                  _p(off, C.c_uint64), _p(ns, C.c_uint32))
+    if used == 2**64 - 1:
+        return mcml_events_batch(p, id0, count, seed, cap * 4)
+    return ev[:used], off, ns
+
+
 def mcml_rsp(p: MCParams) -> float:
     return lib().or_mcml_rsp(C.byref(p))
 
@@ -226,6 +247,17 @@ def ws_loopmerge(nsteps, mode, T, W=32, events=None):
                            n_valid, K, mode, T, C.byref(o))
     else:
         lib().ws_loopmerge(_p(nsteps, C.c_uint32), None, None, W, n_valid, K, mode, T, C.byref(o))
+    return o.as_dict(LM)
+
+
+def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32):
+    """nsteps [n_valid, K]; ev_off [n_valid*K] offsets into the flat event buffer."""
+    nsteps = np.ascontiguousarray(nsteps, np.uint32)
+    ev_off = np.ascontiguousarray(ev_off, np.uint64)
+    n_valid, K = nsteps.shape
+    o = WsCounts()
+    lib().ws_loopmerge(_p(nsteps, C.c_uint32), _p(ev_flat, C.c_uint8), _p(ev_off, C.c_uint64),
+                       W, n_valid, K, mode, T, C.byref(o))
     return o.as_dict(LM)
 
 

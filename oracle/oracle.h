@@ -85,11 +85,17 @@ enum { OR_MC_PHOTONS = 0, OR_MC_STEPS, OR_MC_RD_EXITS, OR_MC_TT_EXITS, OR_MC_RR_
  * NULL) receives the per-photon step count. */
 void or_mcml(const or_mcml_params* p, uint64_t id0, uint64_t count, uint64_t seed,
              uint64_t* A, uint64_t* Rd, uint64_t* Tt, uint64_t* cnt, uint32_t* steps_out);
-/* Per-photon event stream for the simulator (one byte per step):
- * bit0 = boundary (else interaction).  Returns number of steps written
- * (<= cap); stops at cap. */
+/* Per-photon event stream for the simulator (one byte per step) recording
+ * which branches of the step ran (no effect on the arithmetic).  Returns
+ * number of steps written (<= cap); stops at cap. */
+enum { OR_EV_BOUNDARY = 1, OR_EV_SLEFT = 2, OR_EV_REFLECT = 4, OR_EV_EXIT = 8,
+       OR_EV_TRANSMIT = 16, OR_EV_ROULETTE = 32, OR_EV_SPIN_AXIS = 64,
+       OR_EV_SPIN_GENERAL = 128 };
 uint32_t or_mcml_events(const or_mcml_params* p, uint64_t id, uint64_t seed,
                         uint8_t* ev, uint32_t cap);
+uint64_t or_mcml_events_batch(const or_mcml_params* p, uint64_t id0, uint64_t count,
+                              uint64_t seed, uint8_t* ev, uint64_t cap, uint64_t* off,
+                              uint32_t* nsteps);
 /* MCML Fresnel reflectance (all-or-none decision uses it) */
 float or_mcml_fresnel(float ni, float nt, float ca1, float* ca2);
 /* Rsp as defined in mcml.c (specular reflectance at launch) */
@@ -123,8 +129,11 @@ enum { WS_CC_ENTRY = 0, WS_CC_THEN, WS_CC_ELSE_PRE, WS_CC_CALL, WS_CC_ELSE_POST,
        WS_CC_MERGE, WS_CC_NREG };
 /* regions of the loop-merge program (Fig. 2(b), Fig. 3) */
 enum { WS_LM_ENTRY = 0, WS_LM_LAUNCH, WS_LM_STEP, WS_LM_STEP_BOUNDARY,
-       WS_LM_STEP_INTERACT, WS_LM_ROUND, WS_LM_RELEASE, WS_LM_ADVANCE, WS_LM_NREG };
-#define WS_MAX_REG 16
+       WS_LM_STEP_INTERACT, WS_LM_ROUND, WS_LM_RELEASE, WS_LM_ADVANCE,
+       WS_LM_EV0 = 8,      /* .. WS_LM_EV0+7: step lanes whose event has bit b set   */
+       WS_LM_NEV0 = 16,    /* .. WS_LM_NEV0+7: step lanes whose event has bit b clear */
+       WS_LM_NREG = 24 };
+#define WS_MAX_REG 24
 typedef struct {
   uint64_t rounds;                 /* SR scheduler rounds (0 under PDOM) */
   uint64_t execs[WS_MAX_REG];      /* warp-level executions of a region  */

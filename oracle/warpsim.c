@@ -117,13 +117,24 @@ void ws_commoncall(const uint8_t* arm, uint32_t W, uint32_t n_valid, int mode, w
 
 /* ------------------------------------------------------------------ */
 /* Loop Merge: Fig. 2(b), Fig. 3.                */
-static uint32_t step_mask_split(const uint8_t* ev, const uint64_t* ev_off, uint32_t K,
-                                const uint32_t* kk, const uint32_t* jj, uint32_t mask) {
-  uint32_t b = 0;
-  for (uint32_t l = 0; l < 32; ++l)
-    if (mask >> l & 1u)
-      if (ev[ev_off[l * K + kk[l]] + jj[l]] & 1u) b |= 1u << l;
-  return b;
+/* Split one step's mask by the branch outcomes recorded in the event bytes
+ * (bit b set / clear), so every branch of the step body is costed with the
+ * lanes that took it. */
+static void step_split(ws_counts* o, const uint8_t* ev, const uint64_t* ev_off, uint32_t K,
+                       const uint32_t* kk, const uint32_t* jj, uint32_t mask) {
+  uint32_t set[8] = {0};
+  for (uint32_t l = 0; l < 32; ++l) {
+    if (!(mask >> l & 1u)) continue;
+    uint8_t e = ev[ev_off[l * K + kk[l]] + jj[l]];
+    for (int b = 0; b < 8; ++b)
+      if (e >> b & 1u) set[b] |= 1u << l;
+  }
+  hit(o, WS_LM_STEP_BOUNDARY, set[0]);
+  hit(o, WS_LM_STEP_INTERACT, mask & ~set[0]);
+  for (int b = 0; b < 8; ++b) {
+    hit(o, WS_LM_EV0 + b, set[b]);
+    hit(o, WS_LM_NEV0 + b, mask & ~set[b]);
+  }
 }
 
 void ws_loopmerge(const uint32_t* nsteps, const uint8_t* ev, const uint64_t* ev_off, uint32_t W,
@@ -144,9 +155,7 @@ void ws_loopmerge(const uint32_t* nsteps, const uint8_t* ev, const uint64_t* ev_
         if (!m) break;
         hit(o, WS_LM_STEP, m);
         if (ev) {
-          uint32_t b = step_mask_split(ev, ev_off, K, kk, jj, m);
-          hit(o, WS_LM_STEP_BOUNDARY, b);
-          hit(o, WS_LM_STEP_INTERACT, m & ~b);
+          step_split(o, ev, ev_off, K, kk, jj, m);
         }
         for (uint32_t l = 0; l < n_valid; ++l)
           if (m >> l & 1u) jj[l] += 1;
@@ -168,9 +177,7 @@ void ws_loopmerge(const uint32_t* nsteps, const uint8_t* ev, const uint64_t* ev_
       hit(o, WS_LM_RELEASE, P);
       hit(o, WS_LM_STEP, P);
       if (ev) {
-        uint32_t b = step_mask_split(ev, ev_off, K, kk, jj, P);
-        hit(o, WS_LM_STEP_BOUNDARY, b);
-        hit(o, WS_LM_STEP_INTERACT, P & ~b);
+        step_split(o, ev, ev_off, K, kk, jj, P);
       }
       for (uint32_t l = 0; l < n_valid; ++l) {
         if (!(P >> l & 1u)) continue;

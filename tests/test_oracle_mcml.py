@@ -118,6 +118,16 @@ def test_event_stream_matches_step_counts():
     p = P(I.C3)
     o = oracle.mcml(p, 77, 20, 3, steps=True)
     for k in range(20):
-        ev = oracle.mcml_events(p, 77 + k, 3)
+        ev = oracle.mcml_events(p, 77 + k, 3).astype(np.int64)
         assert len(ev) == o["steps"][k]
-        assert set(np.unique(ev)) <= {0, 1}
+        bnd = (ev & oracle.EV_BOUNDARY) != 0
+        outcome = ev & (oracle.EV_REFLECT | oracle.EV_EXIT | oracle.EV_TRANSMIT)
+        spin = ev & (oracle.EV_SPIN_AXIS | oracle.EV_SPIN_GENERAL)
+        # a boundary step has exactly one outcome and no spin; an interaction the reverse
+        assert np.all(np.where(bnd, np.isin(outcome, [4, 8, 16]), outcome == 0))
+        assert np.all(np.where(bnd, spin == 0, np.isin(spin, [64, 128])))
+        # the step after a boundary step resumes the leftover path length
+        assert np.all(((ev[1:] & oracle.EV_SLEFT) != 0) == bnd[:-1])
+        assert (ev[0] & oracle.EV_SLEFT) == 0
+        # only the last step can exit
+        assert np.all((ev[:-1] & oracle.EV_EXIT) == 0)

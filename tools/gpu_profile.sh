@@ -1,14 +1,28 @@
 #!/bin/bash
-# Run under gpurun: bench + ncu evidence for one round. Usage: tools/gpu_profile.sh <tag>
+# Run under gpurun: GPU tests, bench, and the ncu evidence for one round.
+#   bash tools/gpu_profile.sh <tag> [quick]
+# Outputs under gpurun_out/ (summarised into profiles/ by tools/summarize_ncu.py).
 set -x
 TAG=${1:-r01}
 O=gpurun_out
 mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()"
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > $O/gpu_$TAG.txt
+if [ "$2" != "quick" ]; then
+  timeout 1200 python -m pytest tests -m gpu -q > $O/tests_$TAG.log 2>&1; tail -3 $O/tests_$TAG.log
+  timeout 300 python __graft_entry__.py smoke > $O/smoke_$TAG.log 2>&1; tail -1 $O/smoke_$TAG.log
+fi
 timeout 900 python bench.py > $O/bench_$TAG.json 2> $O/bench_$TAG.err
-M=smsp__thread_inst_executed_per_inst_executed.ratio,smsp__inst_executed.sum,smsp__thread_inst_executed.sum,smsp__thread_inst_executed_pred_on.sum,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__cycles_elapsed.avg.per_second,gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,sm__sass_thread_inst_executed_op_ffma_pred_on.sum,smsp__warps_active.avg.pct_of_peak_sustained_active,launch__registers_per_thread,launch__grid_size,launch__block_size
-timeout 900 ncu --metrics $M --clock-control none -k regex:"divloop|commoncall|mcml" --csv --log-file $O/simt_$TAG.csv python tools/one_launch.py > $O/simt_$TAG.log 2>&1
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-configs > $O/launches_$TAG.log 2>&1
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:mcml_spec -c 1 -o $O/prof_mcml_spec_$TAG python tools/one_launch.py mcml --modes spec > $O/prof_$TAG.log 2>&1
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:mcml_pdom -c 1 -o $O/prof_mcml_pdom_$TAG python tools/one_launch.py mcml --modes pdom >> $O/prof_$TAG.log 2>&1
-ls -la $O
+M=smsp__thread_inst_executed_per_inst_executed.ratio,smsp__inst_executed.sum,smsp__thread_inst_executed.sum,smsp__thread_inst_executed_pred_on.sum,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__cycles_elapsed.avg.per_second,gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,sm__sass_thread_inst_executed_op_ffma_pred_on.sum,smsp__warps_active.avg.pct_of_peak_sustained_active,launch__registers_per_thread,launch__grid_size,launch__block_size,lts__t_bytes.sum,l1tex__t_bytes.sum
+# every kernel family at its configs[] size (bench launch configuration)
+timeout 1200 ncu --metrics $M --clock-control none -k regex:"divloop|commoncall|mcml|pt_" --csv --log-file $O/simt_$TAG.csv python tools/one_launch.py > $O/simt_$TAG.log 2>&1
+# the simulator validation launches (static assignment, the oracle replays every warp)
+timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes pdom,spec --threshold 32 > /dev/null 2>&1
+timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic8_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes spec --threshold 8 > /dev/null 2>&1
+# launch list of one short bench run (shares, not absolutes)
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-configs > $O/launches_$TAG.log 2>&1
+# full captures of the dominant kernel (and its PDOM baseline), at 2M photons
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:mcml -c 2 -o $O/prof_mcml_$TAG python tools/one_launch.py mcml --photons 2000000 > $O/prof_$TAG.log 2>&1
+# dram traffic of the bench-sized dominant kernel
+timeout 600 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none -k regex:mcml_spec -c 1 --csv --log-file $O/traffic_$TAG.csv python tools/one_launch.py mcml --modes spec > /dev/null 2>&1
+ls -la $O | tail -30

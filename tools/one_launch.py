@@ -19,6 +19,7 @@ ap.add_argument("--photons", type=int, default=I.C3.n_photons)
 ap.add_argument("--modes", default="pdom,spec")
 ap.add_argument("--threshold", type=int, default=32)
 ap.add_argument("--static", action="store_true")
+ap.add_argument("--iters", type=int, default=0, help="MCML photons per lane (default configs[2]: 64)")
 a = ap.parse_args()
 modes = a.modes.split(",")
 ctx = sr.Context.create(0, 1 << 20)
@@ -38,12 +39,13 @@ if "commoncall" in a.what:
         sr.sr_run(w, c.n_threads, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_CALL, 0)
 if "mcml" in a.what:
     m = I.C3
-    nt = a.photons // m.iters
+    iters = a.iters or m.iters
+    nt = a.photons // iters
     w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
                          flags=sr.F_STATIC if a.static else 0)
     ctx.ensure(sr.sr_workspace_bytes(w, nt))
     for md in modes:
-        sr.sr_run(w, nt, m.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
+        sr.sr_run(w, nt, iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
                   0 if md == "pdom" else a.threshold)
 if "pathtrace" in a.what:
     c = I.C4

@@ -54,15 +54,35 @@ def region_map(path):
     return out
 
 
+def marked_call_lines(path):
+    """Lines that call a __device__ function whose own body carries markers
+    (e.g. the MC step): an instruction resolved only to such a line lost its
+    intermediate inline frames."""
+    src = open(path).read().splitlines()
+    fn, marked = None, set()
+    for line in src:
+        m = re.search(r"__device__[^(;]*?\b(\w+)\s*\(", line)
+        if m and "__global__" not in line:
+            fn = m.group(1)
+        elif "__global__" in line:
+            fn = None
+        if fn and MARK_RE.search(line):
+            marked.add(fn)
+    out = set()
+    for i, line in enumerate(src, 1):
+        code = line.split("//")[0]
+        if any(re.search(r"\b%s\s*\(" % f, code) for f in marked) and "__device__" not in code:
+            out.add(i)
+    return out
+
+
 def extract_cubins(tmp):
     subprocess.run(["cuobjdump", "-xelf", "all", LIB], cwd=tmp, capture_output=True)
     return [os.path.join(tmp, f) for f in os.listdir(tmp) if f.endswith(".cubin")]
 
 
-def parse_functions(cubin):
-    """{function: [dict(addr, text, file, line, outer_file, outer_line, label_before)]}"""
-    txt = subprocess.run(["nvdisasm", "-gi", "-c", cubin], capture_output=True, text=True).stdout
-    funcs, cur, loc, labels = {}, None, (None, None, None, None, []), []
+def _parse(txt):
+    funcs, cur, loc, labels = {}, None, (None, None, []), []
     for raw in txt.splitlines():
         m = re.match(r"\s*\.text\.(\S+):", raw)
         if m:
@@ -74,10 +94,7 @@ def parse_functions(cubin):
         m = LINE_RE.search(raw)
         if m:
             f, ln, rest = m.group(1), int(m.group(2)), m.group(3)
-            inl = INL_RE.findall(rest)
-            of, ol = (inl[-1][0], int(inl[-1][1])) if inl else (f, ln)
-            chain = [(f, ln)] + [(a, int(b)) for a, b in inl]   # innermost -> outermost
-            loc = (f, ln, of, ol, chain)
+            loc = (f, ln, [(f, ln)] + [(a, int(b)) for a, b in INL_RE.findall(rest)])
             continue
         m = re.match(r"^(\.L_x_\d+|\$\S+):$", raw.strip())
         if m:
@@ -86,10 +103,30 @@ def parse_functions(cubin):
         m = INS_RE.search(raw)
         if m:
             funcs[cur].append(dict(addr=int(m.group(1), 16), text=m.group(2), file=loc[0],
-                                   line=loc[1], outer_file=loc[2], outer_line=loc[3],
-                                   chain=loc[4], labels=labels))
+                                   line=loc[1], frames=loc[2], labels=labels))
             labels = []
     return funcs
+
+
+def parse_functions(cubin):
+    """{function: [dict(addr, text, chain, labels)]}.  nvdisasm -g gives the
+    innermost source line of every instruction; -gi adds one 'inlined at'
+    frame (and for deeper inlining reports an outer call site instead), so the
+    chain is the -g frame followed by the -gi frames."""
+    g = _parse(subprocess.run(["nvdisasm", "-g", "-c", cubin], capture_output=True,
+                              text=True).stdout)
+    gi = _parse(subprocess.run(["nvdisasm", "-gi", "-c", cubin], capture_output=True,
+                               text=True).stdout)
+    out = {}
+    for name, ins in g.items():
+        other = gi.get(name, [])
+        for k, x in enumerate(ins):
+            chain = list(x["frames"][:1])
+            if k < len(other) and other[k]["addr"] == x["addr"]:
+                chain += [fr for fr in other[k]["frames"] if fr not in chain]
+            x["chain"] = chain
+        out[name] = ins
+    return out
 
 
 def cold_set(ins):
@@ -140,10 +177,12 @@ def loop_intervals(ins):
 
 
 def kernel_costs(kernel_regex=".*"):
-    maps = {}
+    maps, weak_lines = {}, set()
     for f in os.listdir(CSRC):
         if f.endswith(".cu"):
-            maps[os.path.join(CSRC, f)] = region_map(os.path.join(CSRC, f))
+            path = os.path.join(CSRC, f)
+            maps[path] = region_map(path)
+            weak_lines |= {(path, ln) for ln in marked_call_lines(path)}
     with tempfile.TemporaryDirectory() as tmp:
         funcs = {}
         for c in extract_cubins(tmp):
@@ -170,17 +209,49 @@ def kernel_costs(kernel_regex=".*"):
             sub_size[lb] = len(si) if hot else 0
         cold = cold_set(body)
         loops = [(a, b) for a, b in loop_intervals(body) if a not in cold and b not in cold]
+        # region of each instruction: "strong" when resolved by its own line or
+        # a reported call site; "weak" when only resolved by a line that calls
+        # a marked device function (the intermediate call line was lost).
+        # Weak instructions take the majority strong region of their basic
+        # block (inlined helper code shares the block of its call site).
+        strong, weak = [None] * len(body), [None] * len(body)
+        for i, x in enumerate(body):
+            ch = x["chain"]
+            for j, (f, ln) in enumerate(ch):
+                r = maps.get(f, {}).get(ln)
+                if r is not None:
+                    if j > 0 and (f, ln) in weak_lines:
+                        weak[i] = r
+                    else:
+                        strong[i] = r
+                    break
+        bbs, start = [], 0
+        for i, x in enumerate(body):
+            if i > start and x["labels"]:
+                bbs.append((start, i))
+                start = i
+            if re.match(r"(@!?U?P\w+\s+)?(BRA|EXIT|RET)\b", x["text"]):
+                bbs.append((start, i + 1))
+                start = i + 1
+        if start < len(body):
+            bbs.append((start, len(body)))
+        final, prev = [None] * len(body), None
+        for a_, b_ in bbs:
+            votes = {}
+            for i in range(a_, b_):
+                if strong[i] is not None and i not in cold:
+                    votes[strong[i]] = votes.get(strong[i], 0) + 1
+            bb_reg = max(votes, key=votes.get) if votes else None
+            for i in range(a_, b_):
+                final[i] = strong[i] or bb_reg or prev or weak[i]
+            if bb_reg is not None:
+                prev = bb_reg
         reg = {}
         unmapped = 0
         for i, x in enumerate(body):
             if i in cold:
                 continue
-            # the innermost inline frame that lies in a marked region decides
-            r = None
-            for f, ln in x["chain"]:
-                r = maps.get(f, {}).get(ln)
-                if r is not None:
-                    break
+            r = final[i]
             if r is None:
                 unmapped += 1
                 r = ("UNMAPPED", True)

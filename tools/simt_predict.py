@@ -73,8 +73,22 @@ def commoncall_warps(mode):
         yield oracle.ws_commoncall(a, mode), len(a)
 
 
+MC_VALIDATION = dict(n_threads=16384, iters=8)   # static launch the oracle can replay
+
+
+def mcml_warps(mode, T, n_threads=MC_VALIDATION["n_threads"], iters=MC_VALIDATION["iters"]):
+    m = I.C3
+    p = oracle.mc_params(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap)
+    ev, off, ns = oracle.mcml_events_batch(p, 0, n_threads * iters, I.PRIMARY_SEED)
+    ev = np.ascontiguousarray(ev)
+    for w in range(0, n_threads, 32):
+        lanes = np.arange(w, min(w + 32, n_threads))
+        ids = lanes[:, None] + np.arange(iters)[None, :] * n_threads   # static assignment
+        yield oracle.ws_loopmerge_raw(ns[ids], ev, off[ids].ravel(), mode, T), len(lanes)
+
+
 def main():
-    costs = sass_regions.kernel_costs("divloop_|commoncall_")
+    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_")
     measured = json.load(open(os.path.join(ROOT, "profiles", "simt_efficiency.json")))
     rows = {}
     cases = [
@@ -82,6 +96,9 @@ def main():
         ("divloop_spec(T=16)", r"divloop_specILi125ELb0", lambda: divloop_warps(oracle.SPEC_LOOP, 16)),
         ("commoncall_pdom", r"commoncall_pdomILi250ELb0", lambda: commoncall_warps(oracle.PDOM)),
         ("commoncall_spec", r"commoncall_specILi250ELb0", lambda: commoncall_warps(oracle.SPEC_CALL)),
+        ("mcml_pdom_static", r"mcml_pdomILb0ELb0", lambda: mcml_warps(oracle.PDOM, 0)),
+        ("mcml_spec_static(T=32)", r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 32)),
+        ("mcml_spec_static(T=8)", r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 8)),
     ]
     for label, pat, gen in cases:
         p = predict(find(costs, pat), gen())
