@@ -30,10 +30,10 @@ PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
 DL = dict(ENTRY=0, PROLOG=1, EXPENSIVE=2, EPILOG=3, ROUND=4, RELEASE=5, ADVANCE=6)
 CC = dict(ENTRY=0, THEN=1, ELSE_PRE=2, CALL=3, ELSE_POST=4, MERGE=5)
 LM = dict(ENTRY=0, LAUNCH=1, STEP=2, STEP_BOUNDARY=3, STEP_INTERACT=4, ROUND=5, RELEASE=6,
-          ADVANCE=7, **{f"EV{b}": 8 + b for b in range(8)}, **{f"NEV{b}": 16 + b for b in range(8)})
+          ADVANCE=7, **{f"EV{b}": 8 + b for b in range(16)}, **{f"NEV{b}": 24 + b for b in range(16)})
 # MC step event bits (oracle.h OR_EV_*)
 EV_BOUNDARY, EV_SLEFT, EV_REFLECT, EV_EXIT, EV_TRANSMIT, EV_ROULETTE, EV_SPIN_AXIS, \
-    EV_SPIN_GENERAL = 1, 2, 4, 8, 16, 32, 64, 128
+    EV_SPIN_GENERAL, EV_EXTERNAL = 1, 2, 4, 8, 16, 32, 64, 128, 256
 MC_COUNTERS = ["photons", "steps", "rd_exits", "tt_exits", "rr_kills", "rr_survive", "capped",
                "zero_w"]
 MAX_LAYERS = 8
@@ -61,7 +61,7 @@ class MCParams(C.Structure):
 
 
 class WsCounts(C.Structure):
-    _fields_ = [("rounds", C.c_uint64), ("execs", C.c_uint64 * 24), ("lanes", C.c_uint64 * 24)]
+    _fields_ = [("rounds", C.c_uint64), ("execs", C.c_uint64 * 40), ("lanes", C.c_uint64 * 40)]
 
     def as_dict(self, names):
         return {"rounds": int(self.rounds),
@@ -92,13 +92,13 @@ def lib():
                                     u8p]
         L.or_mcml.argtypes = [C.POINTER(MCParams), C.c_uint64, C.c_uint64, C.c_uint64, u64p, u64p,
                               u64p, u64p, u32p]
-        L.or_mcml_events.argtypes = [C.POINTER(MCParams), C.c_uint64, C.c_uint64, u8p, C.c_uint32]
+        L.or_mcml_events.argtypes = [C.POINTER(MCParams), C.c_uint64, C.c_uint64, C.POINTER(C.c_uint16), C.c_uint32]
         L.or_mcml_events.restype = C.c_uint32
         L.or_mcml_rsp.argtypes = [C.POINTER(MCParams)]; L.or_mcml_rsp.restype = C.c_float
         L.ws_divloop.argtypes = [u8p, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int, C.c_uint32,
                                  C.POINTER(WsCounts)]
         L.ws_commoncall.argtypes = [u8p, C.c_uint32, C.c_uint32, C.c_int, C.POINTER(WsCounts)]
-        L.ws_loopmerge.argtypes = [u32p, u8p, u64p, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int,
+        L.ws_loopmerge.argtypes = [u32p, C.POINTER(C.c_uint16), u64p, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int,
                                    C.c_uint32, C.POINTER(WsCounts)]
         L.ws_divloop_optimum.argtypes = [u8p, C.c_uint32, C.c_uint32]
         L.ws_divloop_optimum.restype = C.c_uint32
@@ -190,23 +190,23 @@ def mcml(p: MCParams, id0, count, seed, steps=False):
 
 
 def mcml_events(p: MCParams, pid, seed, cap=1 << 20):
-    ev = np.zeros(cap, np.uint8)
-    n = lib().or_mcml_events(C.byref(p), pid, seed, _p(ev, C.c_uint8), cap)
+    ev = np.zeros(cap, np.uint16)
+    n = lib().or_mcml_events(C.byref(p), pid, seed, _p(ev, C.c_uint16), cap)
     return ev[:n].copy()
 
 
 def mcml_events_batch(p: MCParams, id0, count, seed, cap=None):
-    """(ev uint8[total], off uint64[count], nsteps uint32[count])"""
+    """(ev uint16[total], off uint64[count], nsteps uint32[count])"""
     L = lib()
     L.or_mcml_events_batch.argtypes = [C.POINTER(MCParams), C.c_uint64, C.c_uint64, C.c_uint64,
-                                       C.POINTER(C.c_uint8), C.c_uint64,
+                                       C.POINTER(C.c_uint16), C.c_uint64,
                                        C.POINTER(C.c_uint64), C.POINTER(C.c_uint32)]
     L.or_mcml_events_batch.restype = C.c_uint64
     cap = cap or count * 2000
-    ev = np.zeros(cap, np.uint8)
+    ev = np.zeros(cap, np.uint16)
     off = np.zeros(count, np.uint64)
     ns = np.zeros(count, np.uint32)
-    used = L.or_mcml_events_batch(C.byref(p), id0, count, seed, _p(ev, C.c_uint8), cap,
+    used = L.or_mcml_events_batch(C.byref(p), id0, count, seed, _p(ev, C.c_uint16), cap,
                                   _p(off, C.c_uint64), _p(ns, C.c_uint32))
     if used == 2**64 - 1:
         return mcml_events_batch(p, id0, count, seed, cap * 4)
@@ -234,7 +234,7 @@ def ws_commoncall(arm, mode, W=32):
 
 
 def ws_loopmerge(nsteps, mode, T, W=32, events=None):
-    """nsteps: [n_valid, K] uint32; events: optional list-of-lists of uint8 arrays."""
+    """nsteps: [n_valid, K] uint32; events: optional list-of-lists of uint16 arrays."""
     nsteps = np.ascontiguousarray(nsteps, np.uint32)
     n_valid, K = nsteps.shape
     o = WsCounts()
@@ -242,8 +242,8 @@ def ws_loopmerge(nsteps, mode, T, W=32, events=None):
         flat = [events[l][k] for l in range(n_valid) for k in range(K)]
         off = np.zeros(len(flat), np.uint64)
         np.cumsum([len(e) for e in flat[:-1]], out=off[1:]) if len(flat) > 1 else None
-        ev = np.ascontiguousarray(np.concatenate(flat) if flat else np.zeros(1), np.uint8)
-        lib().ws_loopmerge(_p(nsteps, C.c_uint32), _p(ev, C.c_uint8), _p(off, C.c_uint64), W,
+        ev = np.ascontiguousarray(np.concatenate(flat) if flat else np.zeros(1), np.uint16)
+        lib().ws_loopmerge(_p(nsteps, C.c_uint32), _p(ev, C.c_uint16), _p(off, C.c_uint64), W,
                            n_valid, K, mode, T, C.byref(o))
     else:
         lib().ws_loopmerge(_p(nsteps, C.c_uint32), None, None, W, n_valid, K, mode, T, C.byref(o))
@@ -256,7 +256,7 @@ def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32):
     ev_off = np.ascontiguousarray(ev_off, np.uint64)
     n_valid, K = nsteps.shape
     o = WsCounts()
-    lib().ws_loopmerge(_p(nsteps, C.c_uint32), _p(ev_flat, C.c_uint8), _p(ev_off, C.c_uint64),
+    lib().ws_loopmerge(_p(nsteps, C.c_uint32), _p(ev_flat, C.c_uint16), _p(ev_off, C.c_uint64),
                        W, n_valid, K, mode, T, C.byref(o))
     return o.as_dict(LM)
 

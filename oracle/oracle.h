@@ -88,13 +88,14 @@ void or_mcml(const or_mcml_params* p, uint64_t id0, uint64_t count, uint64_t see
 /* Per-photon event stream for the simulator (one byte per step) recording
  * which branches of the step ran (no effect on the arithmetic).  Returns
  * number of steps written (<= cap); stops at cap. */
+typedef uint16_t or_event;
 enum { OR_EV_BOUNDARY = 1, OR_EV_SLEFT = 2, OR_EV_REFLECT = 4, OR_EV_EXIT = 8,
        OR_EV_TRANSMIT = 16, OR_EV_ROULETTE = 32, OR_EV_SPIN_AXIS = 64,
-       OR_EV_SPIN_GENERAL = 128 };
+       OR_EV_SPIN_GENERAL = 128, OR_EV_EXTERNAL = 256 /* boundary with the ambient */ };
 uint32_t or_mcml_events(const or_mcml_params* p, uint64_t id, uint64_t seed,
-                        uint8_t* ev, uint32_t cap);
+                        or_event* ev, uint32_t cap);
 uint64_t or_mcml_events_batch(const or_mcml_params* p, uint64_t id0, uint64_t count,
-                              uint64_t seed, uint8_t* ev, uint64_t cap, uint64_t* off,
+                              uint64_t seed, or_event* ev, uint64_t cap, uint64_t* off,
                               uint32_t* nsteps);
 /* MCML Fresnel reflectance (all-or-none decision uses it) */
 float or_mcml_fresnel(float ni, float nt, float ca1, float* ca2);
@@ -130,10 +131,10 @@ enum { WS_CC_ENTRY = 0, WS_CC_THEN, WS_CC_ELSE_PRE, WS_CC_CALL, WS_CC_ELSE_POST,
 /* regions of the loop-merge program (Fig. 2(b), Fig. 3) */
 enum { WS_LM_ENTRY = 0, WS_LM_LAUNCH, WS_LM_STEP, WS_LM_STEP_BOUNDARY,
        WS_LM_STEP_INTERACT, WS_LM_ROUND, WS_LM_RELEASE, WS_LM_ADVANCE,
-       WS_LM_EV0 = 8,      /* .. WS_LM_EV0+7: step lanes whose event has bit b set   */
-       WS_LM_NEV0 = 16,    /* .. WS_LM_NEV0+7: step lanes whose event has bit b clear */
-       WS_LM_NREG = 24 };
-#define WS_MAX_REG 24
+       WS_LM_EV0 = 8,      /* .. WS_LM_EV0+15: step lanes whose event has bit b set   */
+       WS_LM_NEV0 = 24,    /* .. WS_LM_NEV0+15: step lanes whose event has bit b clear */
+       WS_LM_NREG = 40 };
+#define WS_MAX_REG 40
 typedef struct {
   uint64_t rounds;                 /* SR scheduler rounds (0 under PDOM) */
   uint64_t execs[WS_MAX_REG];      /* warp-level executions of a region  */
@@ -148,7 +149,7 @@ void ws_commoncall(const uint8_t* arm, uint32_t W, uint32_t n_valid, int mode, w
 /* Loop merge: lane l owns tasks k < K; task (l,k) runs nsteps[l*K+k] >= 1 inner
  * iterations; ev (may be NULL) gives each step's bit0 = boundary, laid out
  * per task at ev_off[l*K+k]. */
-void ws_loopmerge(const uint32_t* nsteps, const uint8_t* ev, const uint64_t* ev_off,
+void ws_loopmerge(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
                   uint32_t W, uint32_t n_valid, uint32_t K, int mode, uint32_t T,
                   ws_counts* out);
 /* Exhaustive search (tiny warps) of the minimum number of Expensive

@@ -120,24 +120,24 @@ void ws_commoncall(const uint8_t* arm, uint32_t W, uint32_t n_valid, int mode, w
 /* Split one step's mask by the branch outcomes recorded in the event bytes
  * (bit b set / clear), so every branch of the step body is costed with the
  * lanes that took it. */
-static void step_split(ws_counts* o, const uint8_t* ev, const uint64_t* ev_off, uint32_t K,
+static void step_split(ws_counts* o, const or_event* ev, const uint64_t* ev_off, uint32_t K,
                        const uint32_t* kk, const uint32_t* jj, uint32_t mask) {
-  uint32_t set[8] = {0};
+  uint32_t set[16] = {0};
   for (uint32_t l = 0; l < 32; ++l) {
     if (!(mask >> l & 1u)) continue;
-    uint8_t e = ev[ev_off[l * K + kk[l]] + jj[l]];
-    for (int b = 0; b < 8; ++b)
+    or_event e = ev[ev_off[l * K + kk[l]] + jj[l]];
+    for (int b = 0; b < 16; ++b)
       if (e >> b & 1u) set[b] |= 1u << l;
   }
   hit(o, WS_LM_STEP_BOUNDARY, set[0]);
   hit(o, WS_LM_STEP_INTERACT, mask & ~set[0]);
-  for (int b = 0; b < 8; ++b) {
+  for (int b = 0; b < 16; ++b) {
     hit(o, WS_LM_EV0 + b, set[b]);
     hit(o, WS_LM_NEV0 + b, mask & ~set[b]);
   }
 }
 
-void ws_loopmerge(const uint32_t* nsteps, const uint8_t* ev, const uint64_t* ev_off, uint32_t W,
+void ws_loopmerge(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off, uint32_t W,
                   uint32_t n_valid, uint32_t K, int mode, uint32_t T, ws_counts* o) {
   memset(o, 0, sizeof *o);
   if (n_valid > W) n_valid = W;

@@ -1,0 +1,45 @@
+"""The warp simulator (oracle part 2) x static SASS region costs of the built
+cubin predicts each kernel's whole-kernel SIMT efficiency within 2 points of
+the ncu measurement stored in profiles/simt_efficiency.json (BASELINE.json
+north_star: "the simulator-predicted SIMT efficiency must match ncu within 2
+points").  Runs on CPU; the measurement comes from the last gpurun profile of
+the SAME kernel code (per-kernel SASS hash); a stale measurement skips."""
+import json
+import os
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, os.path.join(ROOT, "tools"))
+
+CASES = ["divloop_pdom", "divloop_spec(T=16)", "commoncall_pdom", "commoncall_spec",
+         "mcml_pdom_static", "mcml_spec_static(T=32)", "mcml_spec_static(T=8)"]
+
+
+@pytest.fixture(scope="module")
+def prediction():
+    import __graft_entry__
+    __graft_entry__.build()
+    import sass_regions
+    import simt_predict
+    measured = json.load(open(os.path.join(ROOT, "profiles", "simt_efficiency.json")))
+    hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_")
+    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_")
+    return measured, hashes, costs, simt_predict
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("label", CASES)
+def test_simt_prediction_within_2_points(prediction, label):
+    measured, hashes, costs, sp = prediction
+    m = measured.get(label)
+    if not m or m.get("simt_efficiency") is None:
+        pytest.skip(f"no ncu measurement for {label} in profiles/simt_efficiency.json")
+    if m.get("sass_sha") not in hashes.values():
+        pytest.skip(f"{label}: stored ncu measurement is for different SASS (re-profile)")
+    pattern, gen = sp.CASES[label]
+    p = sp.predict(sp.find(costs, pattern), gen())
+    assert abs(p["simt"] - m["simt_efficiency"]) * 100 < 2.0, (label, p["simt"], m["simt_efficiency"])
+    # the instruction count itself is predicted too
+    assert abs(p["inst"] / m["inst"] - 1) < 0.05, (label, p["inst"], m["inst"])

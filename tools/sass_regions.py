@@ -129,6 +129,21 @@ def parse_functions(cubin):
     return out
 
 
+def basic_blocks(ins):
+    """[start, end) index ranges: a block starts at a label or after a branch."""
+    bbs, start = [], 0
+    for i, x in enumerate(ins):
+        if i > start and x["labels"]:
+            bbs.append((start, i))
+            start = i
+        if re.match(r"(@!?U?P\w+\s+)?(BRA|EXIT|RET)\b", x["text"]):
+            bbs.append((start, i + 1))
+            start = i + 1
+    if start < len(ins):
+        bbs.append((start, len(ins)))
+    return bbs
+
+
 def cold_set(ins):
     """Indices of instructions on cold paths."""
     label_at = {}
@@ -151,7 +166,13 @@ def cold_set(ins):
             if re.match(r"(@\S+\s+)?(RET|BRA)\b", t) and not t.startswith("@"):
                 break
             i += 1
-    # 2. trailing trap loop / padding
+    # 2. the argument/result moves around a call of a cold subroutine (the IEEE
+    #    div/sqrt slow paths): the whole basic block holding the CALL is cold
+    for a, b in basic_blocks(ins):
+        if any(re.search(r"CALL\.\w+(?:\.NOINC)?\s+`\(\$__internal", ins[i]["text"])
+               for i in range(a, b)):
+            cold.update(range(a, b))
+    # 3. trailing trap loop / padding
     for i, x in enumerate(ins):
         m = re.search(r"BRA\s+`\((\.L_x_\d+)\)", x["text"])
         if m and label_at.get(m.group(1)) == i:
@@ -174,6 +195,28 @@ def loop_intervals(ins):
             if j is not None and j < i:
                 out.append((j, i))
     return out
+
+
+def kernel_hashes(kernel_regex=".*"):
+    """{kernel: sha256 of its SASS instruction text} -- identifies the exact
+    code a stored ncu measurement belongs to."""
+    import hashlib
+    with tempfile.TemporaryDirectory() as tmp:
+        out = {}
+        for c in extract_cubins(tmp):
+            txt = subprocess.run(["cuobjdump", "-sass", c], capture_output=True, text=True).stdout
+            cur, buf = None, []
+            for line in txt.splitlines() + ["Function : <end>"]:
+                m = re.search(r"Function : (\S+)", line)
+                if m:
+                    if cur and re.search(kernel_regex, cur):
+                        out[cur] = hashlib.sha256("\n".join(buf).encode()).hexdigest()[:16]
+                    cur, buf = m.group(1), []
+                else:
+                    mm = re.search(r"/\*[0-9a-f]{4,}\*/\s+(.*?);", line)
+                    if mm:
+                        buf.append(mm.group(1).strip())
+        return out
 
 
 def kernel_costs(kernel_regex=".*"):
@@ -243,7 +286,10 @@ def kernel_costs(kernel_regex=".*"):
                     votes[strong[i]] = votes.get(strong[i], 0) + 1
             bb_reg = max(votes, key=votes.get) if votes else None
             for i in range(a_, b_):
-                final[i] = strong[i] or bb_reg or prev or weak[i]
+                # every instruction of a basic block issues with the block's
+                # mask (if-converted code and predicated-off lanes included), so
+                # the block's majority region decides the lanes of all of them
+                final[i] = bb_reg or strong[i] or prev or weak[i]
             if bb_reg is not None:
                 prev = bb_reg
         reg = {}

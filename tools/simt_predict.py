@@ -87,19 +87,22 @@ def mcml_warps(mode, T, n_threads=MC_VALIDATION["n_threads"], iters=MC_VALIDATIO
         yield oracle.ws_loopmerge_raw(ns[ids], ev, off[ids].ravel(), mode, T), len(lanes)
 
 
+CASES = {
+    "divloop_pdom": (r"divloop_pdomILi125ELb0", lambda: divloop_warps(oracle.PDOM, 0)),
+    "divloop_spec(T=16)": (r"divloop_specILi125ELb0", lambda: divloop_warps(oracle.SPEC_LOOP, 16)),
+    "commoncall_pdom": (r"commoncall_pdomILi250ELb0", lambda: commoncall_warps(oracle.PDOM)),
+    "commoncall_spec": (r"commoncall_specILi250ELb0", lambda: commoncall_warps(oracle.SPEC_CALL)),
+    "mcml_pdom_static": (r"mcml_pdomILb0ELb0", lambda: mcml_warps(oracle.PDOM, 0)),
+    "mcml_spec_static(T=32)": (r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 32)),
+    "mcml_spec_static(T=8)": (r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 8)),
+}
+
+
 def main():
     costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_")
     measured = json.load(open(os.path.join(ROOT, "profiles", "simt_efficiency.json")))
     rows = {}
-    cases = [
-        ("divloop_pdom", r"divloop_pdomILi125ELb0", lambda: divloop_warps(oracle.PDOM, 0)),
-        ("divloop_spec(T=16)", r"divloop_specILi125ELb0", lambda: divloop_warps(oracle.SPEC_LOOP, 16)),
-        ("commoncall_pdom", r"commoncall_pdomILi250ELb0", lambda: commoncall_warps(oracle.PDOM)),
-        ("commoncall_spec", r"commoncall_specILi250ELb0", lambda: commoncall_warps(oracle.SPEC_CALL)),
-        ("mcml_pdom_static", r"mcml_pdomILb0ELb0", lambda: mcml_warps(oracle.PDOM, 0)),
-        ("mcml_spec_static(T=32)", r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 32)),
-        ("mcml_spec_static(T=8)", r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 8)),
-    ]
+    cases = [(k, v[0], v[1]) for k, v in CASES.items()]
     for label, pat, gen in cases:
         p = predict(find(costs, pat), gen())
         m = measured.get(label, {})

@@ -35,10 +35,25 @@ def read_ncu_csv(path):
             continue
         if hdr and len(r) == len(hdr):
             d = dict(zip(hdr, r))
-            name = re.sub(r"\(.*", "", d["Kernel Name"]).replace("void sr::<unnamed>::", "")
+            name = re.sub(r"\([^()]*\)$", "", d["Kernel Name"].strip())
+            name = name.replace("void ", "").replace("sr::<unnamed>::", "")
             key = (int(d["ID"]), name)
             data.setdefault(key, {})[d["Metric Name"]] = d["Metric Value"].replace(",", "")
     return [(k[1], v) for k, v in sorted(data.items())]
+
+
+def mangle_match(demangled, mangled):
+    """'divloop_spec<125, false>' vs '_ZN..12divloop_specILi125ELb0EE..'"""
+    m = re.search(r"(\w+)<([^<>]*)>\s*$", demangled.strip())
+    if not m:
+        return False
+    name, args = m.group(1), [a.strip() for a in m.group(2).split(",")]
+    enc = ""
+    for a in args:
+        v = a.replace("(bool)", "").replace("(int)", "").strip()
+        v = {"true": "1", "false": "0"}.get(v, v)
+        enc += r"L[bi]%sE" % re.escape(v)   # ncu may print bools as 0/1
+    return re.search(r"\d" + name + r"I" + enc + r"E", mangled) is not None
 
 
 def num(x):
@@ -78,6 +93,13 @@ def main():
             js[lab] = row_of(kname, m)
     js["_source"] = (f"ncu --metrics ... --clock-control none; tools/one_launch.py; round tag {tag};"
                      " libsr built from this commit")
+    sys.path.insert(0, os.path.join(ROOT, "tools"))
+    import sass_regions
+    hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_|pt_")
+    for lab, r in js.items():
+        if isinstance(r, dict):
+            mangled = [k for k in hashes if mangle_match(r["kernel"], k)]
+            r["sass_sha"] = hashes[mangled[0]] if len(mangled) == 1 else None
     json.dump(js, open(os.path.join(PROF, "simt_efficiency.json"), "w"), indent=1)
     md = [f"# ncu per-kernel summary ({tag})", "",
           "One launch of each kernel (tools/one_launch.py), `ncu --clock-control none`. "
