@@ -95,6 +95,9 @@ typedef struct {
   uint64_t scene_bytes;
   uint32_t width, height; /* image; n_threads must equal width*height           */
   uint32_t max_depth;     /* bounces per path (>= 1)                            */
+  uint32_t merge_unroll;  /* SR_SPEC_LOOP node-granularity merge: BVH node visits
+                             per release round, the partial unroll of P:1467-1474
+                             (0 = 8). Results are identical for every value.   */
 } sr_pathtrace_params;
 
 typedef struct {

@@ -23,6 +23,7 @@ namespace {
 
 struct CallArgs {
   uint64_t t0, n, seed;
+  RoundKeys keys;
   uint32_t iters, split_u32, rounds;
   float* y;
   unsigned long long* counters;
@@ -50,7 +51,7 @@ __global__ void __launch_bounds__(1024) commoncall_pdom(const CallArgs a) {
   float ysum = 0.0f;
   uint32_t then_cnt = 0, execs = 0, lanes = 0;
   for (uint32_t it = 0; it < a.iters; ++it) {  // @sr-region MERGE:full
-    const uint4 u = draw(it, kTagCall, t, a.seed);
+    const uint4 u = draw(it, kTagCall, t, a.keys);
     const float x = u01(u.y);
     float y;
     if (u.x < a.split_u32) {                 // then-arm
@@ -90,7 +91,7 @@ __global__ void __launch_bounds__(1024) commoncall_spec(const CallArgs a) {
   float ysum = 0.0f;
   uint32_t then_cnt = 0, execs = 0, lanes = 0;
   for (uint32_t it = 0; it < a.iters; ++it) {  // @sr-region MERGE:full
-    const uint4 u = draw(it, kTagCall, t, a.seed);
+    const uint4 u = draw(it, kTagCall, t, a.keys);
     const float x = u01(u.y);
     const bool c = u.x < a.split_u32;
     float arg = x;                           // then-arm: argument only
@@ -144,6 +145,7 @@ cudaError_t launch_commoncall(const LaunchCtx& c, const sr_workload& w, uint64_t
   a.t0 = w.task_offset;
   a.n = n;
   a.seed = seed;
+  a.keys = round_keys(seed);
   a.iters = iters;
   a.split_u32 = w.commoncall.split_u32;
   a.rounds = w.commoncall.fma_count / 8u;

@@ -55,7 +55,9 @@ struct PtArgs {
   const PtTri* tris;
   const PtMat* mats;
   uint32_t width, height, spp, max_depth, T;
+  uint32_t unroll;                  // node visits per release (partial unroll)
   uint64_t n, seed;
+  RoundKeys keys;
   float* rgb;                       // 3 floats per pixel
   unsigned long long* counters;     // [0] paths [1] rays [2] node visits [3] tri tests
   uint32_t* sched;
@@ -113,6 +115,11 @@ __device__ __forceinline__ void tri_test(const PtTri& T, V3 o, V3 d, float& tb, 
 // child boxes, the triangles of child leaves, push/pop).  closest_hit() runs
 // it to completion; the node-granularity Loop Merge kernel interleaves single
 // steps of different lanes' rays.
+//
+// The traversal stack lives in shared memory, one column per thread
+// (entry i of thread t at smem[i * blockDim + t]: consecutive lanes hit
+// consecutive banks), so the per-lane traversal state that stays in
+// registers is small and the node fetches have L1 to themselves.
 struct Trav {
   V3 o, d, inv;
   float tb;
@@ -120,8 +127,15 @@ struct Trav {
   uint32_t mb, slot;
   int32_t node;
   int32_t sp;
-  int32_t stack[kStack];
+  int32_t* stk;     // this thread's column of the CTA's shared stack
+  uint32_t stride;  // blockDim.x
 };
+
+__device__ __forceinline__ void trav_bind(Trav& tr) {
+  extern __shared__ int32_t pt_stack_smem[];
+  tr.stk = pt_stack_smem + threadIdx.x;
+  tr.stride = blockDim.x;
+}
 
 __device__ __forceinline__ void trav_begin(Trav& tr, V3 o, V3 d) {
   tr.o = o;
@@ -164,7 +178,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
   if (in0 && in1) {
     const bool first0 = tn0 <= tn1;
     next = first0 ? N.ref0 : N.ref1;
-    if (tr.sp < kStack) tr.stack[tr.sp++] = first0 ? N.ref1 : N.ref0;
+    if (tr.sp < kStack) tr.stk[(tr.sp++) * tr.stride] = first0 ? N.ref1 : N.ref0;
   } else if (in0) {
     next = N.ref0;
   } else if (in1) {
@@ -172,7 +186,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
   }
   if (next < 0) {
     if (tr.sp == 0) return false;
-    next = tr.stack[--tr.sp];
+    next = tr.stk[(--tr.sp) * tr.stride];
   }
   tr.node = next;
   return true;
@@ -193,7 +207,7 @@ struct Path {
 
 __device__ __forceinline__ void camera_ray(const PtArgs& a, const PtHeader& H, Path& p) {
   const uint64_t q = (uint64_t)p.pix * a.spp + p.s;
-  const uint4 u = draw(0u, kTagPt, q, a.seed);
+  const uint4 u = draw(0u, kTagPt, q, a.keys);
   const uint32_t px = p.pix % a.width, py = p.pix / a.width;
   const float fx = ((float)px + u01(u.x)) / (float)a.width;
   const float fy = ((float)py + u01(u.y)) / (float)a.height;
@@ -244,7 +258,7 @@ __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
       const V3 n = entering ? ng : scl(ng, -1.0f);
       const V3 pt = add(p.o, scl(p.d, t));
       const uint64_t q = (uint64_t)p.pix * a.spp + p.s;
-      const uint4 u = draw(p.b + 1u, kTagPt, q, a.seed);
+      const uint4 u = draw(p.b + 1u, kTagPt, q, a.keys);
       if (kind == 0u) {
         const float r1 = u01(u.x);
         const float rr = sqrtf(r1);
@@ -328,6 +342,7 @@ __global__ void __launch_bounds__(128) pt_pdom(const PtArgs a) {
   p.sum = mk(0.0f, 0.0f, 0.0f);
   p.alive = false;
   Trav tr;
+  trav_bind(tr);
   Stats st{0, 0, 0};
   uint32_t paths = 0, outer = 0, rel = 0, rel_lanes = 0, launch_lanes = 0;
   for (uint32_t s = 0; s < a.spp; ++s) {
@@ -368,6 +383,7 @@ __global__ void __launch_bounds__(128) pt_spec(const PtArgs a) {
   p.alive = false;
   p.s = 0;
   Trav tr;
+  trav_bind(tr);
   bool trav = false;                   // NODE: a ray of this lane is being traversed
   Stats st{0, 0, 0};
   uint32_t paths = 0, rounds = 0, rel = 0, rel_lanes = 0, adv = 0, adv_lanes = 0;
@@ -382,7 +398,9 @@ __global__ void __launch_bounds__(128) pt_spec(const PtArgs a) {
       if constexpr (SCHED) { ++rel; rel_lanes += __popc(P); }
       if ((P >> lane_id()) & 1u) {
         __syncwarp(P);
-        if constexpr (NODE) trav = trav_step(a, tr, st);
+        if constexpr (NODE) {
+          for (uint32_t k = 0; k < a.unroll && trav; ++k) trav = trav_step(a, tr, st);
+        }
         else bounce(a, p, tr, st);
       }
     } else {
@@ -413,6 +431,7 @@ __global__ void pt_query(const PtArgs a) {
   const float* r = a.q_rays + 6 * i;
   Stats st{0, 0, 0};
   Trav tr;
+  trav_bind(tr);
   const int64_t h = closest_hit(a, tr, mk(r[0], r[1], r[2]), mk(r[3], r[4], r[5]), st);
   a.q_hit[i] = h;
   a.q_t[i] = tr.tb;
@@ -461,9 +480,11 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
   a.height = w.pathtrace.height;
   a.spp = iters;
   a.max_depth = w.pathtrace.max_depth;
+  a.unroll = w.pathtrace.merge_unroll ? w.pathtrace.merge_unroll : 8;
   a.T = T;
   a.n = n;
   a.seed = seed;
+  a.keys = round_keys(seed);
   a.rgb = reinterpret_cast<float*>(c.ws + c.lay.off[SR_T_PERTHREAD]);
   a.counters = reinterpret_cast<unsigned long long*>(c.ws + c.lay.off[SR_T_COUNTERS]);
   a.sched = (w.flags & SR_F_SCHED) ? reinterpret_cast<uint32_t*>(c.ws + c.lay.off[SR_T_SCHED])
@@ -471,19 +492,29 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
   const uint32_t block = c.block;
   const uint64_t grid = (n + block - 1) / block;
   if (grid > 0x7fffffffull) return cudaErrorInvalidConfiguration;
-  record_launch((uint32_t)grid, block, 0);
   const bool spec = mode == SR_SPEC_LOOP;
   const bool node = (w.flags & SR_F_COARSE) == 0;
   const unsigned gr = (unsigned)grid;
+  const size_t smem = (size_t)kStack * block * sizeof(int32_t);  // traversal stacks
+  if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
+  record_launch((uint32_t)grid, block, (uint32_t)smem);
+  if (smem > 48 * 1024) {
+    cudaFuncSetAttribute(pt_pdom<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_pdom<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  }
   if (!spec) {
-    if (a.sched) pt_pdom<true><<<gr, block, 0, c.stream>>>(a);
-    else pt_pdom<false><<<gr, block, 0, c.stream>>>(a);
+    if (a.sched) pt_pdom<true><<<gr, block, smem, c.stream>>>(a);
+    else pt_pdom<false><<<gr, block, smem, c.stream>>>(a);
   } else if (node) {
-    if (a.sched) pt_spec<true, true><<<gr, block, 0, c.stream>>>(a);
-    else pt_spec<false, true><<<gr, block, 0, c.stream>>>(a);
+    if (a.sched) pt_spec<true, true><<<gr, block, smem, c.stream>>>(a);
+    else pt_spec<false, true><<<gr, block, smem, c.stream>>>(a);
   } else {
-    if (a.sched) pt_spec<true, false><<<gr, block, 0, c.stream>>>(a);
-    else pt_spec<false, false><<<gr, block, 0, c.stream>>>(a);
+    if (a.sched) pt_spec<true, false><<<gr, block, smem, c.stream>>>(a);
+    else pt_spec<false, false><<<gr, block, smem, c.stream>>>(a);
   }
   return cudaGetLastError();
 }
@@ -503,7 +534,7 @@ cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* ray
   a.q_t = t;
   const unsigned grid = (unsigned)((n + 127) / 128);
   record_launch(grid, 128, 0);
-  if (n) pt_query<<<grid, 128, 0, st>>>(a);
+  if (n) pt_query<<<grid, 128, kStack * 128 * sizeof(int32_t), st>>>(a);
   return cudaGetLastError();
 }
 

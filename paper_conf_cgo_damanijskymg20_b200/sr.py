@@ -59,7 +59,7 @@ class MCMLParams(C.Structure):
 
 class PathtraceParams(C.Structure):
     _fields_ = [("scene_dev", C.c_void_p), ("scene_bytes", C.c_uint64), ("width", C.c_uint32),
-                ("height", C.c_uint32), ("max_depth", C.c_uint32)]
+                ("height", C.c_uint32), ("max_depth", C.c_uint32), ("merge_unroll", C.c_uint32)]
 
 
 class Workload(C.Structure):
@@ -217,9 +217,9 @@ def upload_scene(tris, mat, mats, cam, device: int = 0):
 
 
 def pathtrace_workload(scene_ptr: int, scene_bytes: int, width: int, height: int, max_depth=8,
-                       flags=0, block=0) -> Workload:
+                       flags=0, block=0, unroll=0) -> Workload:
     w = Workload(kind=WL_PATHTRACE, flags=flags, block_threads=block)
-    w.pathtrace = PathtraceParams(scene_ptr, scene_bytes, width, height, max_depth)
+    w.pathtrace = PathtraceParams(scene_ptr, scene_bytes, width, height, max_depth, unroll)
     return w
 
 

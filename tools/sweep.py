@@ -24,6 +24,7 @@ ap.add_argument("--blocks", default="0")
 ap.add_argument("--photons", type=int, default=I.C3.n_photons)
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--flags", type=int, default=0, help="extra sr_workload.flags (e.g. 4 = F_COARSE)")
+ap.add_argument("--unroll", type=int, default=0, help="PT node-merge partial unroll")
 a = ap.parse_args()
 Ts = [int(x) for x in a.thresholds.split(",")]
 blocks = [int(x) for x in a.blocks.split(",")]
@@ -101,7 +102,7 @@ if "pathtrace" in a.what:
     res = []
     for b in blocks:
         w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth, block=b,
-                                  flags=a.flags)
+                                  flags=a.flags, unroll=a.unroll)
         ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
             t = timed(lambda: sr.sr_run(w, c.n_pixels, c.spp, seed, mode, T), a.reps)
