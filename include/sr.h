@@ -56,7 +56,8 @@ typedef enum {
   SR_WL_DIVLOOP = 0,     /* Fig. 2(a): divergent condition in a loop (config 1) */
   SR_WL_COMMONCALL = 1,  /* Fig. 2(c): common function call          (config 2) */
   SR_WL_MCML = 2,        /* Fig. 2(b): MC photon transport, loop merge (3, 5)  */
-  SR_WL_PATHTRACE = 3    /* Fig. 2(b): path tracer, loop merge       (config 4) */
+  SR_WL_PATHTRACE = 3,   /* Fig. 2(b): path tracer, loop merge       (config 4) */
+  SR_WL_RSBENCH = 4      /* Fig. 3: RSBench-shaped nested trip-count loop (NEXT-1) */
 } sr_workload_kind;
 
 /* sr_workload.flags */
@@ -101,6 +102,11 @@ typedef struct {
 } sr_pathtrace_params;
 
 typedef struct {
+  uint32_t fma_count;  /* FMAs of the per-nuclide body; multiple of 8 (64)       */
+  uint32_t reserved;   /* must be 0                                              */
+} sr_rsbench_params;   /* materials / nuclide counts: DESIGN.md reading R8       */
+
+typedef struct {
   int32_t kind;            /* sr_workload_kind                                   */
   uint32_t flags;          /* SR_F_*                                             */
   uint64_t task_offset;    /* global id of this caller's first task (sharding)  */
@@ -110,6 +116,7 @@ typedef struct {
   sr_commoncall_params commoncall;
   sr_mcml_params mcml;
   sr_pathtrace_params pathtrace;
+  sr_rsbench_params rsbench;
 } sr_workload;
 
 /* Bind the context to a device, a stream and a caller-owned device

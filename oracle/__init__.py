@@ -20,7 +20,7 @@ import numpy as np
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB = os.path.join(HERE, "liboracle.so")
 SOURCES = ["philox.c", "srmath.c", "divloop.c", "commoncall.c", "mcml.c", "warpsim.c",
-           "pathtrace.c"]
+           "pathtrace.c", "rsbench.c"]
 CFLAGS = ["-O2", "-std=gnu11", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
           "-Wall", "-Wno-unused-function"]
 
@@ -161,6 +161,31 @@ def commoncall(t0, n, iters, seed, split_u32=1 << 31, fma_count=2000):
     lib().or_commoncall(_p(prm, C.c_uint32), t0, n, iters, seed, _p(y, C.c_float),
                         _p(arm, C.c_uint8))
     return y, arm
+
+
+# ---------------------------------------------------------------- NEXT-1 (RSBench shape)
+RS_MATS, RS_NUCLIDES = 12, 355
+
+
+def rsbench(t0, n, iters, seed, fma_count=64, trips=False):
+    L = lib()
+    u32p, f32p = C.POINTER(C.c_uint32), C.POINTER(C.c_float)
+    L.or_rsbench.argtypes = [C.c_uint32, C.c_uint64, C.c_uint64, C.c_uint32, C.c_uint64, f32p,
+                             u32p, u32p]
+    acc = np.zeros(n, np.float32); nuc = np.zeros(n, np.uint32)
+    tr = np.zeros(n * iters, np.uint32) if trips else None
+    L.or_rsbench(fma_count, t0, n, iters, seed, _p(acc, C.c_float), _p(nuc, C.c_uint32),
+                 _p(tr, C.c_uint32) if trips else None)
+    return (acc, nuc, tr.reshape(n, iters)) if trips else (acc, nuc)
+
+
+def rs_table():
+    L = lib()
+    L.or_rs_nuclides.restype = C.c_uint32; L.or_rs_nuclides.argtypes = [C.c_uint32]
+    L.or_rs_threshold.restype = C.c_uint32; L.or_rs_threshold.argtypes = [C.c_uint32]
+    L.or_rs_pick.restype = C.c_uint32; L.or_rs_pick.argtypes = [C.c_uint32]
+    return ([L.or_rs_nuclides(m) for m in range(RS_MATS)],
+            [L.or_rs_threshold(m) for m in range(RS_MATS)], L.or_rs_pick)
 
 
 # ---------------------------------------------------------------- configs 3/5

@@ -120,6 +120,19 @@ void or_pt_render(const or_pt_scene* sc, uint32_t width, uint32_t height, uint32
                   uint32_t max_depth, uint64_t seed, const uint32_t* pixels, uint32_t n_pixels,
                   float* rgb, uint64_t* counters);
 
+/* ---- rsbench.c : NEXT-1, RSBench-shaped nested trip-count loop (Fig. 3). */
+enum { OR_TAG_RS = 5 };
+#define OR_RS_MATS 12
+#define OR_RS_NUCLIDES 355
+uint32_t or_rs_nuclides(uint32_t m);   /* nuclides of material m            */
+uint32_t or_rs_threshold(uint32_t m);  /* cumulative 2^-32 selection bound   */
+uint32_t or_rs_pick(uint32_t u);       /* material of a Philox word          */
+float or_rs_body(float E, uint32_t nuc, uint32_t fma_count);
+/* per thread: acc = sum over lookups of sum over nuclides of body(); nuc =
+ * nuclides visited; trips[j*iters+k] (may be NULL) = inner trip count */
+void or_rsbench(uint32_t fma_count, uint64_t t0, uint64_t n, uint32_t iters, uint64_t seed,
+                float* acc, uint32_t* nuc, uint32_t* trips);
+
 /* ---- warpsim.c : lane-mask warp simulator (oracle part 2). */
 enum { WS_PDOM = 0, WS_SPEC_LOOP = 1, WS_SPEC_CALL = 2 };
 /* regions of the divloop program (Listing 1) */

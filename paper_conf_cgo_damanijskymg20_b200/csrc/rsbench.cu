@@ -1,0 +1,190 @@
+// rsbench.cu -- NEXT-1: the RSBench-shaped nested trip-count loop that the
+// paper uses to introduce Loop Merge (Fig. 3):
+//
+//   for (k = 0; k < lookups_per_thread; k++) {            // coarsened outer loop
+//     Prolog: material m = pick(), energy E                // 12 materials
+//     for (i = 0; i < nuclides(m); i++) L1: xs += body()  // 4 .. 321 trips
+//     Epilog: acc += xs
+//   }
+//
+//   rs_pdom  as written: the warp's inner loop runs until the lane with the
+//            most nuclides is done ("threads that exit the inner loop early
+//            wait for all threads").
+//   rs_spec  Loop Merge + soft barrier: lanes whose inner loop ended run their
+//            epilog and the next lookup's prolog while the others continue, as
+//            in Fig. 3(b)(iii); the inner body runs with the lanes that have
+//            nuclides left once popc >= T (or nobody can refill).
+// One lane = one thread of the problem (static); the lookup order and the
+// nuclide order of each lane are program order, so the float sums are
+// schedule-free (reading R8).
+#include <cmath>
+
+#include "sr_device.cuh"
+#include "sr_internal.h"
+
+namespace sr {
+namespace {
+
+constexpr uint32_t kMats = 12, kNuclides = 355;
+__constant__ uint32_t c_nucs[kMats] = {321, 5, 4, 4, 27, 21, 21, 21, 21, 21, 9, 9};
+
+struct RsArgs {
+  uint64_t t0, n;
+  RoundKeys keys;
+  uint32_t thr[kMats];   // cumulative selection thresholds (host-computed)
+  uint32_t iters, rounds, T;
+  uint2* out;            // {acc bits, nuclides}
+  unsigned long long* counters;
+  uint32_t* sched;
+};
+
+__device__ __forceinline__ uint32_t pick(const RsArgs& a, uint32_t u) {
+  uint32_t m = kMats - 1;
+#pragma unroll
+  for (int i = kMats - 2; i >= 0; --i)
+    if (u < a.thr[i]) m = (uint32_t)i;
+  return m;
+}
+
+template <int ROUNDS>
+__device__ __forceinline__ float body(float E, uint32_t m, uint32_t i, uint32_t rounds) {
+  const uint32_t nuc = (37u * m + 13u * i) % kNuclides;
+  const float start = E + (float)nuc * 0x1p-9f;
+  return expensive<ROUNDS>(start, rounds);
+}
+
+__device__ __forceinline__ void finish(const RsArgs& a, uint64_t g, bool valid, float acc,
+                                       uint32_t nucs, uint32_t rounds, uint32_t rel,
+                                       uint32_t rel_lanes, uint32_t adv, uint32_t adv_lanes) {
+  if (valid) a.out[g] = make_uint2(__float_as_uint(acc), nucs);
+  const uint32_t tot = __reduce_add_sync(kFull, valid ? nucs : 0u);
+  if (lane_id() == 0) {
+    atomicAdd(a.counters, (unsigned long long)tot);
+    if (a.sched) {
+      uint4* p = reinterpret_cast<uint4*>(a.sched + (g >> 5) * kSchedWords);
+      p[0] = make_uint4(rounds, rel, rel_lanes, adv);
+      p[1] = make_uint4(adv_lanes, 0u, 0u, 0u);
+    }
+  }
+}
+
+template <int ROUNDS, bool SCHED>
+__global__ void __launch_bounds__(256) rs_pdom(const RsArgs a) {
+  const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
+  const bool valid = g < a.n;
+  const uint64_t t = a.t0 + g;
+  float acc = 0.0f;
+  uint32_t nucs = 0, rel = 0, rel_lanes = 0;
+  for (uint32_t k = 0; k < a.iters; ++k) {  // @sr-region LAUNCH:full
+    uint32_t N = 0, m = 0;
+    float E = 0.0f;
+    if (valid) {
+      const uint4 u = draw(k, kTagRs, t, a.keys);  // @sr-region LAUNCH
+      m = pick(a, u.x);
+      E = u01(u.y);
+      N = c_nucs[m];
+    }
+    float xs = 0.0f;
+    for (uint32_t i = 0; i < N; ++i) {  // @sr-region STEP
+      if constexpr (SCHED) {
+        const uint32_t mk = __activemask();
+        if (lane_id() == (uint32_t)(__ffs(mk) - 1)) { ++rel; rel_lanes += __popc(mk); }
+      }
+      xs = xs + body<ROUNDS>(E, m, i, a.rounds);
+    }
+    acc = acc + xs;  // @sr-region LAUNCH:full
+    nucs += N;
+  }
+  uint32_t r = 0, rl = 0;  // @sr-region ENTRY:full
+  if constexpr (SCHED) { r = __reduce_add_sync(kFull, rel); rl = __reduce_add_sync(kFull, rel_lanes); }
+  finish(a, g, valid, acc, nucs, a.iters, r, rl, a.iters, a.iters * (uint32_t)__popc(__ballot_sync(kFull, valid)));
+}  // @sr-region END
+
+template <int ROUNDS, bool SCHED>
+__global__ void __launch_bounds__(256) rs_spec(const RsArgs a) {
+  const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
+  const bool valid = g < a.n;
+  const uint64_t t = a.t0 + g;
+  float acc = 0.0f, xs = 0.0f, E = 0.0f;
+  uint32_t nucs = 0, k = 0, i = 0, N = 0, m = 0;
+  bool busy = false;                       // inside a lookup's inner loop
+  uint32_t rounds = 0, rel = 0, rel_lanes = 0, adv = 0, adv_lanes = 0;
+  uint32_t E_mask = __ballot_sync(kFull, !valid || a.iters == 0);  // nothing left (Cancel)
+  for (;;) {
+    const uint32_t P = __ballot_sync(kFull, busy);  // @sr-region ROUND:full
+    const uint32_t R = ~(P | E_mask);
+    if ((P | R) == 0u) break;
+    if constexpr (SCHED) ++rounds;
+    if ((uint32_t)__popc(P) >= a.T || R == 0u) {
+      if constexpr (SCHED) { ++rel; rel_lanes += __popc(P); }  // @sr-region RELEASE:full
+      if (busy) {
+        __syncwarp(P);  // @sr-region STEP
+        xs = xs + body<ROUNDS>(E, m, i, a.rounds);
+        i = i + 1u;
+        if (i == N) {                      // inner loop done: Epilog
+          acc = acc + xs;
+          nucs += N;
+          busy = false;
+        }
+      }
+    } else {
+      if constexpr (SCHED) { ++adv; adv_lanes += __popc(R); }  // @sr-region ADVANCE:full
+      if ((R >> lane_id()) & 1u) {
+        const uint4 u = draw(k, kTagRs, t, a.keys);  // @sr-region LAUNCH
+        m = pick(a, u.x);
+        E = u01(u.y);
+        N = c_nucs[m];
+        i = 0;
+        xs = 0.0f;
+        busy = true;
+        ++k;
+      }
+      E_mask = __ballot_sync(kFull, !valid || k >= a.iters);  // @sr-region ADVANCE:full
+    }
+  }
+  finish(a, g, valid, acc, nucs, rounds, rel, rel_lanes, adv, adv_lanes);  // @sr-region ENTRY:full
+}  // @sr-region END
+
+template <bool SCHED>
+cudaError_t launch_t(const LaunchCtx& c, const RsArgs& a, int mode) {
+  const uint32_t block = c.block;
+  const uint64_t grid = (a.n + block - 1) / block;
+  if (grid > 0x7fffffffull) return cudaErrorInvalidConfiguration;
+  record_launch((uint32_t)grid, block, 0);
+  const bool spec = mode == SR_SPEC_LOOP;
+#define SR_RS(R)                                                                    \
+  (spec ? rs_spec<R, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a)            \
+        : rs_pdom<R, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a))
+  if (a.rounds == 8) SR_RS(8);
+  else SR_RS(0);
+#undef SR_RS
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_rsbench(const LaunchCtx& c, const sr_workload& w, uint64_t n, uint32_t iters,
+                           uint64_t seed, int mode, uint32_t T) {
+  // cumulative selection thresholds floor(2^32 * sum_{i<=m} p_i), last = 2^32-1
+  static const double prob[kMats] = {0.140, 0.052, 0.275, 0.134, 0.154, 0.064,
+                                     0.066, 0.055, 0.008, 0.015, 0.025, 0.013};
+  RsArgs a;
+  double cum = 0.0;
+  for (uint32_t mm = 0; mm < kMats; ++mm) {
+    cum += prob[mm];
+    a.thr[mm] = mm + 1 == kMats ? 0xFFFFFFFFu : (uint32_t)std::floor(cum * 4294967296.0);
+  }
+  a.t0 = w.task_offset;
+  a.n = n;
+  a.keys = round_keys(seed);
+  a.iters = iters;
+  a.rounds = w.rsbench.fma_count / 8u;
+  a.T = T;
+  a.out = reinterpret_cast<uint2*>(c.ws + c.lay.off[SR_T_PERTHREAD]);
+  a.counters = reinterpret_cast<unsigned long long*>(c.ws + c.lay.off[SR_T_COUNTERS]);
+  a.sched = (w.flags & SR_F_SCHED) ? reinterpret_cast<uint32_t*>(c.ws + c.lay.off[SR_T_SCHED])
+                                   : nullptr;
+  return a.sched ? launch_t<true>(c, a, mode) : launch_t<false>(c, a, mode);
+}
+
+}  // namespace sr

@@ -62,6 +62,11 @@ std::string check_workload(const sr_workload* w, uint64_t n_threads) {
       return check_mcml(w->mcml);
     case SR_WL_PATHTRACE:
       return check_pathtrace(w->pathtrace, n_threads);
+    case SR_WL_RSBENCH:
+      if (w->rsbench.fma_count % 8 != 0) return "rsbench.fma_count must be a multiple of 8";
+      if (w->rsbench.reserved != 0) return "rsbench.reserved must be 0";
+      if (n_threads > (1ull << 40)) return "n_threads too large";
+      return "";
     default:
       return "unknown workload kind " + std::to_string(w->kind);
   }
@@ -73,6 +78,7 @@ uint32_t default_block(const sr_workload& w) {
     case SR_WL_DIVLOOP: return 64;
     case SR_WL_COMMONCALL: return 256;
     case SR_WL_MCML: return 512;
+    case SR_WL_RSBENCH: return 256;
     default: return 128;
   }
 }
@@ -93,6 +99,7 @@ Layout layout_of(const sr_workload& w, uint64_t n) {
   size_t per = 0, grid = 0;
   switch (w.kind) {
     case SR_WL_DIVLOOP: per = 8 * n; break;
+    case SR_WL_RSBENCH: per = 8 * n; break;
     case SR_WL_COMMONCALL: per = 4 * n; break;
     case SR_WL_MCML: grid = 8ull * ((uint64_t)w.mcml.nz * w.mcml.nr + 2ull * w.mcml.nr); break;
     case SR_WL_PATHTRACE: per = pathtrace_perthread_bytes(n); break;
@@ -255,6 +262,7 @@ int sr_run(const sr_workload* w, uint64_t n_threads, uint32_t iters, uint64_t se
     case SR_WL_DIVLOOP: e = launch_divloop(c, *w, n_threads, iters, seed, mode, T); break;
     case SR_WL_COMMONCALL: e = launch_commoncall(c, *w, n_threads, iters, seed, mode); break;
     case SR_WL_MCML: e = launch_mcml(c, *w, n_threads, iters, seed, mode, T); break;
+    case SR_WL_RSBENCH: e = launch_rsbench(c, *w, n_threads, iters, seed, mode, T); break;
     default: e = launch_pathtrace(c, *w, n_threads, iters, seed, mode, T); break;
   }
   if (e != cudaSuccess) return fail_cuda(e, "sr_run: kernel launch");

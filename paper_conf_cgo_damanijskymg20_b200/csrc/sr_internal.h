@@ -42,6 +42,8 @@ cudaError_t launch_commoncall(const LaunchCtx& c, const sr_workload& w, uint64_t
                               uint32_t iters, uint64_t seed, int mode);
 cudaError_t launch_mcml(const LaunchCtx& c, const sr_workload& w, uint64_t n, uint32_t iters,
                         uint64_t seed, int mode, uint32_t T);
+cudaError_t launch_rsbench(const LaunchCtx& c, const sr_workload& w, uint64_t n, uint32_t iters,
+                           uint64_t seed, int mode, uint32_t T);
 cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t n,
                              uint32_t iters, uint64_t seed, int mode, uint32_t T);
 

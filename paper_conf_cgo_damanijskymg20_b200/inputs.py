@@ -33,6 +33,19 @@ class CommonCall:
     fma_count: int = 2000
 
 
+@dataclass(frozen=True)
+class RSBench:
+    """NEXT-1: RSBench-shaped nested trip-count loop (Fig. 3).
+    Materials / nuclide counts / selection probabilities: DESIGN.md R8."""
+    n_threads: int = 131072
+    iters: int = 32             # lookups per thread (thread coarsening, P:346-359)
+    fma_count: int = 64         # FMAs of the per-nuclide body
+    threshold: int = 16
+
+
+NEXT1 = RSBench()
+
+
 # (n, mua [1/cm], mus [1/cm], g, d [cm]) -- a synthetic 3-layer tissue slab
 THREE_LAYER = ((1.4, 4.0, 96.0, 0.80, 0.01),
                (1.4, 1.0, 199.0, 0.90, 0.10),

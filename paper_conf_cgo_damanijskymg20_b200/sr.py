@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(HERE, "libsr.so")
 
 SR_OK, SR_E_INVALID, SR_E_STATE, SR_E_NOMEM, SR_E_CUDA = 0, -1, -2, -3, -4
 PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
-WL_DIVLOOP, WL_COMMONCALL, WL_MCML, WL_PATHTRACE = 0, 1, 2, 3
+WL_DIVLOOP, WL_COMMONCALL, WL_MCML, WL_PATHTRACE, WL_RSBENCH = 0, 1, 2, 3, 4
 F_SCHED, F_STATIC, F_COARSE = 1, 2, 4
 T_PERTHREAD, T_GRID, T_COUNTERS, T_SCHED, T_SCRATCH = 0, 1, 2, 3, 4
 MAX_LAYERS = 8
@@ -62,11 +62,16 @@ class PathtraceParams(C.Structure):
                 ("height", C.c_uint32), ("max_depth", C.c_uint32), ("merge_unroll", C.c_uint32)]
 
 
+class RsbenchParams(C.Structure):
+    _fields_ = [("fma_count", C.c_uint32), ("reserved", C.c_uint32)]
+
+
 class Workload(C.Structure):
     _fields_ = [("kind", C.c_int32), ("flags", C.c_uint32), ("task_offset", C.c_uint64),
                 ("block_threads", C.c_uint32), ("grid_ctas", C.c_uint32),
                 ("divloop", DivloopParams), ("commoncall", CommoncallParams),
-                ("mcml", MCMLParams), ("pathtrace", PathtraceParams)]
+                ("mcml", MCMLParams), ("pathtrace", PathtraceParams),
+                ("rsbench", RsbenchParams)]
 
 
 _lib = None
@@ -182,6 +187,12 @@ def sr_scene_build(tris, mat, mats, cam, dst_ptr: int | None, dst_bytes: int) ->
 def divloop_workload(p_u32=1 << 29, fma_count=1000, task_offset=0, flags=0, block=0) -> Workload:
     w = Workload(kind=WL_DIVLOOP, flags=flags, task_offset=task_offset, block_threads=block)
     w.divloop = DivloopParams(p_u32, fma_count)
+    return w
+
+
+def rsbench_workload(fma_count=64, task_offset=0, flags=0, block=0) -> Workload:
+    w = Workload(kind=WL_RSBENCH, flags=flags, task_offset=task_offset, block_threads=block)
+    w.rsbench = RsbenchParams(fma_count, 0)
     return w
 
 

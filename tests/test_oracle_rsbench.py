@@ -1,0 +1,61 @@
+"""Pins of the oracle's RSBench-shaped workload (NEXT-1, Fig. 3):
+material selection frequencies, trip-count statistics, the body's closed
+form, and per-thread sums within the closed-form range."""
+import math
+
+import numpy as np
+
+import oracle
+from paper_conf_cgo_damanijskymg20_b200 import inputs as I
+from tests.test_oracle_microbench import expensive_closed_form, expensive_tol
+
+PROB = [0.140, 0.052, 0.275, 0.134, 0.154, 0.064, 0.066, 0.055, 0.008, 0.015, 0.025, 0.013]
+NUCS = [321, 5, 4, 4, 27, 21, 21, 21, 21, 21, 9, 9]
+
+
+def test_material_table_and_pick_boundaries():
+    nucs, thr, pick = oracle.rs_table()
+    assert nucs == NUCS and min(nucs) == 4 and max(nucs) == 321   # "4 to 321"
+    assert all(a < b for a, b in zip(thr, thr[1:])) and thr[-1] == 2**32 - 1
+    assert abs(thr[0] - 0.140 * 2**32) <= 1
+    for m in range(11):
+        assert pick(thr[m] - 1) == m and pick(thr[m]) == m + 1
+    assert pick(0) == 0 and pick(2**32 - 1) == 11
+
+
+def test_trip_count_distribution():
+    c = I.NEXT1
+    n, iters = 20000, 8
+    _, nuc, trips = oracle.rsbench(0, n, iters, I.PRIMARY_SEED, fma_count=0, trips=True)
+    assert np.array_equal(trips.sum(1), nuc)
+    vals, counts = np.unique(trips, return_counts=True)
+    assert set(vals) <= set(NUCS)
+    # chi^2 of the material frequencies (materials with equal trip counts merged)
+    exp = {}
+    for p, k in zip(PROB, NUCS):
+        exp[k] = exp.get(k, 0.0) + p
+    N = trips.size
+    chi2 = sum((counts[list(vals).index(k)] - N * p) ** 2 / (N * p) for k, p in exp.items())
+    assert chi2 < len(exp) + 5 * math.sqrt(2 * len(exp))
+    mean = sum(p * k for p, k in zip(PROB, NUCS))
+    assert abs(trips.mean() - mean) < 5 * trips.std() / math.sqrt(N)
+
+
+def test_body_closed_form():
+    L = oracle.lib()
+    import ctypes as C
+    L.or_rs_body.argtypes = [C.c_float, C.c_uint32, C.c_uint32]
+    L.or_rs_body.restype = C.c_float
+    for E in (0.0, 0.3, 0.9):
+        for nuc in (0, 17, 354):
+            start = np.float32(np.float32(E) + np.float32(nuc * 2.0**-9))
+            got = L.or_rs_body(E, nuc, 64)
+            assert abs(got - expensive_closed_form(float(start), 64)) <= expensive_tol(64)
+
+
+def test_thread_sums_within_closed_form_range():
+    acc, nuc = oracle.rsbench(0, 500, 4, 3, fma_count=64)
+    lo = expensive_closed_form(0.0, 64) - expensive_tol(64)
+    hi = expensive_closed_form(1.0 + 354 * 2.0**-9, 64) + expensive_tol(64)
+    per = acc / nuc
+    assert per.min() >= lo * (1 - 1e-5) and per.max() <= hi * (1 + 1e-5)

@@ -14,7 +14,8 @@ from paper_conf_cgo_damanijskymg20_b200 import inputs as I  # noqa: E402
 from paper_conf_cgo_damanijskymg20_b200 import sr  # noqa: E402
 
 ap = argparse.ArgumentParser()
-ap.add_argument("what", nargs="*", default=["divloop", "commoncall", "mcml", "pathtrace"])
+ap.add_argument("what", nargs="*", default=["divloop", "commoncall", "mcml", "pathtrace",
+                                             "rsbench"])
 ap.add_argument("--photons", type=int, default=I.C3.n_photons)
 ap.add_argument("--modes", default="pdom,spec")
 ap.add_argument("--threshold", type=int, default=32)
@@ -47,6 +48,13 @@ if "mcml" in a.what:
     for md in modes:
         sr.sr_run(w, nt, iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
                   0 if md == "pdom" else a.threshold)
+if "rsbench" in a.what:
+    c = I.NEXT1
+    w = sr.rsbench_workload(c.fma_count)
+    ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
+    for md in modes:
+        sr.sr_run(w, c.n_threads, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
+                  0 if md == "pdom" else c.threshold)
 if "pathtrace" in a.what:
     c = I.C4
     tris, mat, mats, cam = I.cornell_scene(c)

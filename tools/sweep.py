@@ -95,6 +95,20 @@ if "divloop" in a.what:
             res.append(r)
             print(json.dumps(r), file=sys.stderr, flush=True)
     out["divloop"] = res
+if "rsbench" in a.what:
+    c = I.NEXT1
+    res = []
+    for b in blocks:
+        w = sr.rsbench_workload(c.fma_count, block=b)
+        ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
+        for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
+            t = timed(lambda: sr.sr_run(w, c.n_threads, c.iters, seed, mode, T), a.reps)
+            r = dict(block=b, mode="pdom" if mode == sr.PDOM else "spec", T=T, ms=t,
+                     lookups_per_s=c.n_threads * c.iters / (t * 1e-3), launch=sr.sr_last_launch())
+            r.update(eff(w, c.n_threads, c.iters, mode, T))
+            res.append(r)
+            print(json.dumps(r), file=sys.stderr, flush=True)
+    out["rsbench"] = res
 if "pathtrace" in a.what:
     c = I.C4
     tris, mat, mats, cam = I.cornell_scene(c)
