@@ -405,6 +405,17 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
     res["speedup_vs_pdom"] = res["spec_call"]["value"] / res["pdom"]["value"]
     out["commoncall"] = res
 
+    # NEXT-1: RSBench-shaped nested trip-count loop (Fig. 3), PDOM vs Loop Merge
+    c = I.NEXT1
+    w = sr.rsbench_workload(c.fma_count)
+    res = {}
+    for name, mode, thr in (("pdom", sr.PDOM, 0), (f"spec_t{c.threshold}", sr.SPEC_LOOP,
+                                                   c.threshold)):
+        t = graph_time(w, c.n_threads, c.iters, mode, thr, reps=5)
+        res[name] = {"value": c.n_threads * c.iters / (t * 1e-3), "unit": "lookups/s", "ms": t}
+    res["speedup_vs_pdom"] = res[f"spec_t{c.threshold}"]["value"] / res["pdom"]["value"]
+    out["rsbench"] = res
+
     # configs[3]: path tracer, 1024^2 x 16 spp over the 1,044,494-triangle BVH scene
     c = I.C4
     tris, mat, mats, cam = I.cornell_scene(c)

@@ -85,6 +85,7 @@ __global__ void __launch_bounds__(256) rs_pdom(const RsArgs a) {
       N = c_nucs[m];
     }
     float xs = 0.0f;
+#pragma unroll 1  // one body per trip, as written (an unrolled remainder would split trips)
     for (uint32_t i = 0; i < N; ++i) {  // @sr-region STEP
       if constexpr (SCHED) {
         const uint32_t mk = __activemask();

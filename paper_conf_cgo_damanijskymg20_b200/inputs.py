@@ -40,7 +40,7 @@ class RSBench:
     n_threads: int = 131072
     iters: int = 32             # lookups per thread (thread coarsening)
     fma_count: int = 64         # FMAs of the per-nuclide body
-    threshold: int = 16
+    threshold: int = 24         # best of the sweep (profiles/threshold_sweep_*.md)
 
 
 NEXT1 = RSBench()

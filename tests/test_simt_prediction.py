@@ -14,6 +14,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, os.path.join(ROOT, "tools"))
 
 CASES = ["divloop_pdom", "divloop_spec(T=16)", "commoncall_pdom", "commoncall_spec",
+         "rs_pdom", "rs_spec(T=24)",
          "mcml_pdom_static", "mcml_spec_static(T=32)", "mcml_spec_static(T=8)"]
 
 
@@ -24,8 +25,8 @@ def prediction():
     import sass_regions
     import simt_predict
     measured = json.load(open(os.path.join(ROOT, "profiles", "simt_efficiency.json")))
-    hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_")
-    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_")
+    hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_|rs_")
+    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_|rs_")
     return measured, hashes, costs, simt_predict
 
 

@@ -87,6 +87,14 @@ def mcml_warps(mode, T, n_threads=MC_VALIDATION["n_threads"], iters=MC_VALIDATIO
         yield oracle.ws_loopmerge_raw(ns[ids], ev, off[ids].ravel(), mode, T), len(lanes)
 
 
+def rsbench_warps(mode, T):
+    c = I.NEXT1
+    _, _, trips = oracle.rsbench(0, c.n_threads, c.iters, I.PRIMARY_SEED, fma_count=0, trips=True)
+    for w in range(0, c.n_threads, 32):
+        tr = trips[w:w + 32]
+        yield oracle.ws_loopmerge(tr, mode, T), len(tr)
+
+
 CASES = {
     "divloop_pdom": (r"divloop_pdomILi125ELb0", lambda: divloop_warps(oracle.PDOM, 0)),
     "divloop_spec(T=16)": (r"divloop_specILi125ELb0", lambda: divloop_warps(oracle.SPEC_LOOP, 16)),
@@ -95,11 +103,13 @@ CASES = {
     "mcml_pdom_static": (r"mcml_pdomILb0ELb0", lambda: mcml_warps(oracle.PDOM, 0)),
     "mcml_spec_static(T=32)": (r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 32)),
     "mcml_spec_static(T=8)": (r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 8)),
+    "rs_pdom": (r"rs_pdomILi8ELb0", lambda: rsbench_warps(oracle.PDOM, 0)),
+    "rs_spec(T=24)": (r"rs_specILi8ELb0", lambda: rsbench_warps(oracle.SPEC_LOOP, 24)),
 }
 
 
 def main():
-    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_")
+    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_|rs_")
     measured = json.load(open(os.path.join(ROOT, "profiles", "simt_efficiency.json")))
     rows = {}
     cases = [(k, v[0], v[1]) for k, v in CASES.items()]

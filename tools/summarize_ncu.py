@@ -21,7 +21,8 @@ PROF = os.path.join(ROOT, "profiles")
 
 # launch order of tools/one_launch.py (default: every family, pdom then spec)
 LABELS_ALL = ["divloop_pdom", "divloop_spec(T=16)", "commoncall_pdom", "commoncall_spec",
-              "mcml_pdom", "mcml_spec(T=32)", "pt_pdom", "pt_spec(T=32)"]
+              "mcml_pdom", "mcml_spec(T=32)", "rs_pdom", "rs_spec(T=24)", "pt_pdom",
+              "pt_spec(T=8)"]
 LABELS_MCSTATIC = ["mcml_pdom_static", "mcml_spec_static(T=32)"]
 LABELS_MCSTATIC8 = ["mcml_spec_static(T=8)"]
 
@@ -95,7 +96,7 @@ def main():
                      " libsr built from this commit")
     sys.path.insert(0, os.path.join(ROOT, "tools"))
     import sass_regions
-    hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_|pt_")
+    hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_|pt_|rs_")
     for lab, r in js.items():
         if isinstance(r, dict):
             mangled = [k for k in hashes if mangle_match(r["kernel"], k)]
