@@ -47,6 +47,7 @@ def parse():
     ap.add_argument("--threshold", type=int, default=32)
     ap.add_argument("--photons-per-gpu", type=int, default=0,
                     help="override the per-rank photon count (default: configs[2] = 10^7)")
+    ap.add_argument("--block", type=int, default=0, help="MCML CTA size (0 = library default)")
     ap.add_argument("--no-configs", action="store_true", help="skip the microbenchmark lines")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     return ap.parse_args()
@@ -222,7 +223,7 @@ def main():
     per_rank = nt * iters
     T = args.threshold
     w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
-                         task_offset=P.task_offset_of(rank, per_rank))
+                         task_offset=P.task_offset_of(rank, per_rank), block=args.block)
     nbytes = sr.sr_workspace_bytes(w, nt)
     ctx = sr.Context.create(local, nbytes, stream)
     off, tb = sr.sr_workspace_region(w, nt, sr.T_GRID)

@@ -89,6 +89,12 @@ typedef struct {
   float dr, dz;            /* tally grid spacing, cm                             */
   uint32_t nr, nz;         /* tally grid size (nr, nz >= 1)                      */
   uint32_t step_cap;       /* a photon dies after this many steps (>= 1)         */
+  uint32_t defer_threshold;  /* SR_SPEC_LOOP only: 0 = off; T_b in [1,32] = nest an
+                                Iteration Delay of the boundary sub-step (Fresnel /
+                                transmit / exit) inside the Loop Merge: parked
+                                boundary lanes run together once T_b have arrived
+                                (two concurrent predictions).  Results
+                                are identical for every value.                    */
 } sr_mcml_params;
 
 typedef struct {

@@ -30,7 +30,8 @@ PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
 DL = dict(ENTRY=0, PROLOG=1, EXPENSIVE=2, EPILOG=3, ROUND=4, RELEASE=5, ADVANCE=6)
 CC = dict(ENTRY=0, THEN=1, ELSE_PRE=2, CALL=3, ELSE_POST=4, MERGE=5)
 LM = dict(ENTRY=0, LAUNCH=1, STEP=2, STEP_BOUNDARY=3, STEP_INTERACT=4, ROUND=5, RELEASE=6,
-          ADVANCE=7, **{f"EV{b}": 8 + b for b in range(16)}, **{f"NEV{b}": 24 + b for b in range(16)})
+          ADVANCE=7, **{f"EV{b}": 8 + b for b in range(16)}, **{f"NEV{b}": 24 + b for b in range(16)},
+          A_RR=40, B_RR=41, B_REL=42)
 # MC step event bits (oracle.h OR_EV_*)
 EV_BOUNDARY, EV_SLEFT, EV_REFLECT, EV_EXIT, EV_TRANSMIT, EV_ROULETTE, EV_SPIN_AXIS, \
     EV_SPIN_GENERAL, EV_EXTERNAL = 1, 2, 4, 8, 16, 32, 64, 128, 256
@@ -61,7 +62,7 @@ class MCParams(C.Structure):
 
 
 class WsCounts(C.Structure):
-    _fields_ = [("rounds", C.c_uint64), ("execs", C.c_uint64 * 40), ("lanes", C.c_uint64 * 40)]
+    _fields_ = [("rounds", C.c_uint64), ("execs", C.c_uint64 * 48), ("lanes", C.c_uint64 * 48)]
 
     def as_dict(self, names):
         return {"rounds": int(self.rounds),
@@ -283,6 +284,21 @@ def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32):
     o = WsCounts()
     lib().ws_loopmerge(_p(nsteps, C.c_uint32), _p(ev_flat, C.c_uint16), _p(ev_off, C.c_uint64),
                        W, n_valid, K, mode, T, C.byref(o))
+    return o.as_dict(LM)
+
+
+def ws_loopmerge_defer_raw(nsteps, ev_flat, ev_off, T, Tb, W=32):
+    """Loop Merge + nested Iteration Delay of the boundary sub-step."""
+    nsteps = np.ascontiguousarray(nsteps, np.uint32)
+    ev_off = np.ascontiguousarray(ev_off, np.uint64)
+    n_valid, K = nsteps.shape
+    o = WsCounts()
+    L = lib()
+    L.ws_loopmerge_defer.argtypes = [C.POINTER(C.c_uint32), C.POINTER(C.c_uint16),
+                                     C.POINTER(C.c_uint64), C.c_uint32, C.c_uint32, C.c_uint32,
+                                     C.c_uint32, C.c_uint32, C.POINTER(WsCounts)]
+    L.ws_loopmerge_defer(_p(nsteps, C.c_uint32), _p(ev_flat, C.c_uint16), _p(ev_off, C.c_uint64),
+                         W, n_valid, K, T, Tb, C.byref(o))
     return o.as_dict(LM)
 
 

@@ -146,8 +146,11 @@ enum { WS_LM_ENTRY = 0, WS_LM_LAUNCH, WS_LM_STEP, WS_LM_STEP_BOUNDARY,
        WS_LM_STEP_INTERACT, WS_LM_ROUND, WS_LM_RELEASE, WS_LM_ADVANCE,
        WS_LM_EV0 = 8,      /* .. WS_LM_EV0+15: step lanes whose event has bit b set   */
        WS_LM_NEV0 = 24,    /* .. WS_LM_NEV0+15: step lanes whose event has bit b clear */
-       WS_LM_NREG = 40 };
-#define WS_MAX_REG 40
+       WS_LM_A_RR = 40,    /* deferred mode: roulette of interaction steps (part A)   */
+       WS_LM_B_RR = 41,    /* deferred mode: roulette of boundary steps (part B)      */
+       WS_LM_B_REL = 42,   /* deferred mode: boundary releases, lanes = parked set    */
+       WS_LM_NREG = 43 };
+#define WS_MAX_REG 48
 typedef struct {
   uint64_t rounds;                 /* SR scheduler rounds (0 under PDOM) */
   uint64_t execs[WS_MAX_REG];      /* warp-level executions of a region  */
@@ -162,6 +165,10 @@ void ws_commoncall(const uint8_t* arm, uint32_t W, uint32_t n_valid, int mode, w
 /* Loop merge: lane l owns tasks k < K; task (l,k) runs nsteps[l*K+k] >= 1 inner
  * iterations; ev (may be NULL) gives each step's bit0 = boundary, laid out
  * per task at ev_off[l*K+k]. */
+/* Loop Merge + nested Iteration Delay of the boundary sub-step (warpsim.c) */
+void ws_loopmerge_defer(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
+                        uint32_t W, uint32_t n_valid, uint32_t K, uint32_t T, uint32_t Tb,
+                        ws_counts* out);
 void ws_loopmerge(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
                   uint32_t W, uint32_t n_valid, uint32_t K, int mode, uint32_t T,
                   ws_counts* out);

@@ -198,6 +198,105 @@ void ws_loopmerge(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev
 }
 
 /* ------------------------------------------------------------------ */
+/* Loop Merge with a second, nested prediction: Iteration Delay of the rare
+ * boundary sub-step (two concurrent predictions).  A step is
+ * split into part A (draw, path length, boundary distance; the interaction
+ * branch runs to completion, a boundary hit only moves the photon to the
+ * boundary and parks it) and part B (the boundary's Fresnel / transmit /
+ * exit / roulette, run later for all parked lanes together).  Per round:
+ *   B = parked, P = live and not parked, R = idle lanes with tasks left;
+ *   |B| >= Tb -> boundary release; else |P| >= T -> step release;
+ *   else R != {} -> advance; else P != {} -> step release; else B != {} ->
+ *   boundary release; else exit.
+ * Only the boundary bit (bit0) of the events decides the schedule; the other
+ * bits split each phase's mask for costing: phase A counts bits 1, 6, 7 and
+ * the interaction roulette; phase B counts bits 2, 3, 4, 8 and its roulette. */
+static or_event evt(const or_event* ev, const uint64_t* ev_off, uint32_t K, const uint32_t* kk,
+                    const uint32_t* jj, uint32_t l) {
+  return ev[ev_off[l * K + kk[l]] + jj[l]];
+}
+
+void ws_loopmerge_defer(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
+                        uint32_t W, uint32_t n_valid, uint32_t K, uint32_t T, uint32_t Tb,
+                        ws_counts* o) {
+  memset(o, 0, sizeof *o);
+  if (n_valid > W) n_valid = W;
+  if (T == 0 || T > 32) T = 32;
+  if (Tb == 0 || Tb > 32) Tb = 32;
+  uint32_t valid = n_valid >= 32 ? 0xffffffffu : ((1u << n_valid) - 1u);
+  uint32_t kk[32] = {0}, jj[32] = {0}, next[32] = {0};
+  uint32_t alive = 0, parked = 0;
+  hit(o, WS_LM_ENTRY, valid);
+  for (;;) {
+    uint32_t Bm = parked, P = alive & ~parked, R = 0;
+    for (uint32_t l = 0; l < n_valid; ++l)
+      if (!(alive >> l & 1u) && next[l] < K) R |= 1u << l;
+    if (!Bm && !P && !R) break;
+    o->rounds += 1;
+    hit(o, WS_LM_ROUND, valid);
+    int phase;  /* 1 step release, 2 boundary release, 3 advance */
+    if ((uint32_t)__builtin_popcount(Bm) >= Tb) phase = 2;
+    else if ((uint32_t)__builtin_popcount(P) >= T) phase = 1;
+    else if (R) phase = 3;
+    else if (P) phase = 1;
+    else phase = 2;
+    if (phase == 1) {
+      hit(o, WS_LM_RELEASE, P);
+      hit(o, WS_LM_STEP, P);
+      uint32_t bit[16] = {0};
+      for (uint32_t l = 0; l < n_valid; ++l) {
+        if (!(P >> l & 1u)) continue;
+        or_event e = evt(ev, ev_off, K, kk, jj, l);
+        for (int b = 0; b < 16; ++b)
+          if (e >> b & 1u) bit[b] |= 1u << l;
+      }
+      hit(o, WS_LM_EV0, bit[0]);
+      hit(o, WS_LM_NEV0, P & ~bit[0]);
+      hit(o, WS_LM_EV0 + 1, bit[1]);
+      hit(o, WS_LM_NEV0 + 1, P & ~bit[1]);
+      hit(o, WS_LM_EV0 + 6, bit[6]);
+      hit(o, WS_LM_EV0 + 7, bit[7]);
+      hit(o, WS_LM_A_RR, bit[5] & ~bit[0]);
+      for (uint32_t l = 0; l < n_valid; ++l) {
+        if (!(P >> l & 1u)) continue;
+        if (bit[0] >> l & 1u) { parked |= 1u << l; continue; }   /* Join + Wait */
+        jj[l] += 1;
+        if (jj[l] == nsteps[l * K + kk[l]]) alive &= ~(1u << l);
+      }
+    } else if (phase == 2) {
+      hit(o, WS_LM_B_REL, Bm);
+      uint32_t bit[16] = {0};
+      for (uint32_t l = 0; l < n_valid; ++l) {
+        if (!(Bm >> l & 1u)) continue;
+        or_event e = evt(ev, ev_off, K, kk, jj, l);
+        for (int b = 0; b < 16; ++b)
+          if (e >> b & 1u) bit[b] |= 1u << l;
+      }
+      hit(o, WS_LM_EV0 + 2, bit[2]);
+      hit(o, WS_LM_EV0 + 3, bit[3]);
+      hit(o, WS_LM_EV0 + 4, bit[4]);
+      hit(o, WS_LM_EV0 + 8, bit[8]);
+      hit(o, WS_LM_B_RR, bit[5]);
+      for (uint32_t l = 0; l < n_valid; ++l) {
+        if (!(Bm >> l & 1u)) continue;
+        jj[l] += 1;
+        if (jj[l] == nsteps[l * K + kk[l]]) alive &= ~(1u << l);
+      }
+      parked = 0;
+    } else {
+      hit(o, WS_LM_ADVANCE, R);
+      hit(o, WS_LM_LAUNCH, R);
+      for (uint32_t l = 0; l < n_valid; ++l) {
+        if (!(R >> l & 1u)) continue;
+        kk[l] = next[l]++;
+        jj[l] = 0;
+        alive |= 1u << l;
+      }
+    }
+  }
+}
+
+/* ------------------------------------------------------------------ */
 /* Exhaustive optimum of the iteration-delay program for W <= 4, L <= 4:
  * 0-1 BFS over (it[l], parked[l]); advancing one free lane costs 0,
  * releasing any non-empty subset of parked lanes costs 1 Expensive execution. */

@@ -237,6 +237,37 @@ def test_mcml_schedule_matches_simulator(ctx, mode, T):
             assert g[0] == s["rounds"] and (g[3], g[4]) == s["LAUNCH"], wi
 
 
+@pytest.mark.parametrize("flags", [0, sr.F_STATIC])
+@pytest.mark.parametrize("T,Tb", [(32, 1), (32, 8), (16, 4), (32, 32)])
+def test_mcml_deferred_boundary_bit_exact(ctx, flags, T, Tb):
+    m = I.C3
+    nt, it = 300, 5
+    ref = mc_oracle(m, 0, nt * it, 17)
+    got = run_mc(ctx, mc_workload(m, flags=flags, block=128, defer=Tb), nt, it, 17,
+                 sr.SPEC_LOOP, T, m)
+    assert_mc_equal(got, ref)
+
+
+@pytest.mark.parametrize("T,Tb", [(32, 8), (16, 4), (32, 32)])
+def test_mcml_deferred_schedule_matches_simulator(ctx, T, Tb):
+    m = I.C3
+    nt, it = 96, 6
+    w = mc_workload(m, flags=sr.F_STATIC | sr.F_SCHED, block=32, defer=Tb)
+    run_mc(ctx, w, nt, it, 3, sr.SPEC_LOOP, T, m)
+    sched = ctx.region(w, nt, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    p = oracle.mc_params(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap)
+    ev, off, ns = oracle.mcml_events_batch(p, 0, nt * it, 3)
+    for wi in range(nt // 32):
+        lanes = np.arange(32 * wi, 32 * wi + 32)
+        ids = lanes[:, None] + np.arange(it)[None, :] * nt
+        s = oracle.ws_loopmerge_defer_raw(ns[ids], ev, off[ids].ravel(), T, Tb)
+        g = sched[wi]
+        assert g[0] == s["rounds"], wi
+        assert (g[1], g[2]) == s["STEP"], wi
+        assert (g[3], g[4]) == s["LAUNCH"], wi
+        assert (g[5], g[6]) == s["B_REL"], wi
+
+
 def test_mcml_full_size_invariants(ctx):
     """Config 3 at full size in the bench launch configuration: PDOM == SPEC
     (T=32, 16) bit for bit, == the sum of two shards, and a slice far into the

@@ -131,3 +131,35 @@ def test_loopmerge_event_split_sums_to_step():
     for mode, T in ((PDOM, 0), (SPEC_LOOP, 32), (SPEC_LOOP, 8)):
         r = oracle.ws_loopmerge(n, mode, T, events=ev)
         assert r["STEP_BOUNDARY"][1] + r["STEP_INTERACT"][1] == r["STEP"][1] == n.sum()
+
+
+def _mc_events(K, W, seed):
+    p = oracle.mc_params(I.C3.layers)
+    ev, off, ns = oracle.mcml_events_batch(p, 0, W * K, seed)
+    ids = np.arange(W)[:, None] + np.arange(K)[None, :] * W
+    return ev, off, ns, ids
+
+
+@pytest.mark.parametrize("T,Tb", [(32, 32), (32, 4), (16, 8), (1, 1)])
+def test_loopmerge_defer_conservation(T, Tb):
+    K, W = 4, 32
+    ev, off, ns, ids = _mc_events(K, W, 9)
+    r = oracle.ws_loopmerge_defer_raw(ns[ids], ev, off[ids].ravel(), T, Tb)
+    nb = int(((ev & oracle.EV_BOUNDARY) != 0).sum())
+    assert r["STEP"][1] == ns.sum()                   # every step runs part A once
+    assert r["B_REL"][1] == nb                        # every boundary sub-step runs once
+    assert r["EV0"][1] == nb                          # ... after parking in part A
+    assert r["NEV0"][1] == ns.sum() - nb
+    assert r["LAUNCH"][1] == W * K
+    # the parked set is released in fewer executions than boundary steps
+    assert r["B_REL"][0] <= max(nb, 1)
+
+
+def test_loopmerge_defer_groups_boundaries():
+    """Deferral raises the boundary code's active lanes per execution."""
+    K, W = 8, 32
+    ev, off, ns, ids = _mc_events(K, W, 4)
+    plain = oracle.ws_loopmerge_raw(ns[ids], ev, off[ids].ravel(), oracle.SPEC_LOOP, 32)
+    defer = oracle.ws_loopmerge_defer_raw(ns[ids], ev, off[ids].ravel(), 32, 8)
+    eff = lambda x: x[1] / max(1, 32 * x[0])
+    assert eff(defer["B_REL"]) > 4 * eff(plain["STEP_BOUNDARY"])

@@ -1,0 +1,17 @@
+"""Build tuning variants of libsr next to the product library (SR_LIB selects one)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_cgo_damanijskymg20_b200 import build as B  # noqa: E402
+
+VARIANTS = {
+    "libsr_t640.so": ["SR_MCML_MAXT=640", "SR_MCML_MINB=2"],
+    "libsr_t768.so": ["SR_MCML_MAXT=768", "SR_MCML_MINB=2"],
+    "libsr_t1024.so": ["SR_MCML_MAXT=1024", "SR_MCML_MINB=1"],
+    "libsr_t384.so": ["SR_MCML_MAXT=384", "SR_MCML_MINB=3"],
+}
+if __name__ == "__main__":
+    names = sys.argv[1:] or list(VARIANTS)
+    for n in names:
+        print(B.build(force=True, defines=VARIANTS[n], lib=os.path.join(B.HERE, n)))

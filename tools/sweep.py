@@ -25,6 +25,7 @@ ap.add_argument("--photons", type=int, default=I.C3.n_photons)
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--flags", type=int, default=0, help="extra sr_workload.flags (e.g. 4 = F_COARSE)")
 ap.add_argument("--unroll", type=int, default=0, help="PT node-merge partial unroll")
+ap.add_argument("--defer", type=int, default=0, help="MCML boundary defer threshold T_b")
 a = ap.parse_args()
 Ts = [int(x) for x in a.thresholds.split(",")]
 blocks = [int(x) for x in a.blocks.split(",")]
@@ -68,7 +69,7 @@ if "mcml" in a.what:
     res = []
     for b in blocks:
         w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
-                             block=b)
+                             block=b, defer=a.defer)
         ctx.ensure(sr.sr_workspace_bytes(w, nt))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
             t = timed(lambda: sr.sr_run(w, nt, m.iters, seed, mode, T), a.reps)
