@@ -48,6 +48,8 @@ def parse():
     ap.add_argument("--photons-per-gpu", type=int, default=0,
                     help="override the per-rank photon count (default: configs[2] = 10^7)")
     ap.add_argument("--block", type=int, default=0, help="MCML CTA size (0 = library default)")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo: test the N>1 plumbing on one GPU (ranks share it)")
     ap.add_argument("--no-configs", action="store_true", help="skip the microbenchmark lines")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     return ap.parse_args()
@@ -209,8 +211,14 @@ def main():
     from paper_conf_cgo_damanijskymg20_b200 import sr
 
     ws_n, rank, local = dist_env()
+    if args.dist_backend == "gloo":
+        # plumbing check of the multi-rank path with fewer GPUs than ranks
+        local = local % max(1, torch.cuda.device_count())
     if ws_n > 1:
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        else:
+            dist.init_process_group("gloo")
     torch.cuda.set_device(local)
     dev = torch.device(f"cuda:{local}")
     stream = torch.cuda.Stream(device=dev)
@@ -321,7 +329,8 @@ def main():
                        "threshold": T, "mode": "SPEC_LOOP", "seed": I.PRIMARY_SEED,
                        "l2": "flushed (256 MB write) between timed steps",
                        "launch": launch_spec, "launch_pdom": launch_pdom,
-                       "parallelism": f"dp{ws_n} (photon-id shards + 1 NCCL int64 all-reduce)"},
+                       "parallelism": f"dp{ws_n} (photon-id shards + 1 "
+                                      f"{args.dist_backend.upper()} int64 all-reduce)"},
             "pdom": {"value": pdom_value, "unit": UNIT, "ms_per_step": t_pdom},
             "speedup_vs_pdom": value / pdom_value,
             "common_region_efficiency": {"pdom": eff_pdom, "spec": eff_spec,
