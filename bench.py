@@ -48,6 +48,8 @@ def parse():
     ap.add_argument("--photons-per-gpu", type=int, default=0,
                     help="override the per-rank photon count (default: configs[2] = 10^7)")
     ap.add_argument("--block", type=int, default=0, help="MCML CTA size (0 = library default)")
+    ap.add_argument("--unroll", type=int, default=0,
+                    help="MCML steps per release (0 = inputs.C3.merge_unroll)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: test the N>1 plumbing on one GPU (ranks share it)")
     ap.add_argument("--no-configs", action="store_true", help="skip the microbenchmark lines")
@@ -231,7 +233,8 @@ def main():
     per_rank = nt * iters
     T = args.threshold
     w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
-                         task_offset=P.task_offset_of(rank, per_rank), block=args.block)
+                         task_offset=P.task_offset_of(rank, per_rank), block=args.block,
+                         unroll=args.unroll if args.unroll else m.merge_unroll)
     nbytes = sr.sr_workspace_bytes(w, nt)
     ctx = sr.Context.create(local, nbytes, stream)
     off, tb = sr.sr_workspace_region(w, nt, sr.T_GRID)
@@ -290,7 +293,7 @@ def main():
     def region_eff(mode, thr):
         wi = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz,
                               m.step_cap, task_offset=P.task_offset_of(rank, per_rank),
-                              flags=sr.F_SCHED)
+                              flags=sr.F_SCHED)   # U = 1: lanes per merged-loop iteration
         ctx.ensure(sr.sr_workspace_bytes(wi, nt))
         ni = min(nt, 32768)
         sr.sr_run(wi, ni, iters, I.PRIMARY_SEED, mode, thr)
@@ -327,6 +330,7 @@ def main():
             "config": {"workload": "mcml-3layer (configs[2] per GPU; N GPUs = configs[4] weak-scaled)",
                        "photons_per_gpu": per_rank, "lanes": nt, "photons_per_lane": iters,
                        "threshold": T, "mode": "SPEC_LOOP", "seed": I.PRIMARY_SEED,
+                       "merge_unroll": args.unroll if args.unroll else m.merge_unroll,
                        "l2": "flushed (256 MB write) between timed steps",
                        "launch": launch_spec, "launch_pdom": launch_pdom,
                        "parallelism": f"dp{ws_n} (photon-id shards + 1 "

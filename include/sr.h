@@ -95,6 +95,9 @@ typedef struct {
                                 boundary lanes run together once T_b have arrived
                                 (two concurrent predictions).  Results
                                 are identical for every value.                    */
+  uint32_t merge_unroll;   /* SR_SPEC_LOOP: photon steps per release round, the
+                              partial unroll of the merged loop;
+                              0 = 1.  Results are identical for every value.    */
 } sr_mcml_params;
 
 typedef struct {

@@ -276,14 +276,20 @@ def ws_loopmerge(nsteps, mode, T, W=32, events=None):
     return o.as_dict(LM)
 
 
-def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32):
-    """nsteps [n_valid, K]; ev_off [n_valid*K] offsets into the flat event buffer."""
+def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32, U=1):
+    """nsteps [n_valid, K]; ev_off [n_valid*K] offsets into the flat event buffer;
+    U = steps per release (partial unroll of the merged loop)."""
     nsteps = np.ascontiguousarray(nsteps, np.uint32)
     ev_off = np.ascontiguousarray(ev_off, np.uint64)
     n_valid, K = nsteps.shape
     o = WsCounts()
-    lib().ws_loopmerge(_p(nsteps, C.c_uint32), _p(ev_flat, C.c_uint16), _p(ev_off, C.c_uint64),
-                       W, n_valid, K, mode, T, C.byref(o))
+    L = lib()
+    L.ws_loopmerge_unrolled.argtypes = [C.POINTER(C.c_uint32), C.POINTER(C.c_uint16),
+                                        C.POINTER(C.c_uint64), C.c_uint32, C.c_uint32,
+                                        C.c_uint32, C.c_int, C.c_uint32, C.c_uint32,
+                                        C.POINTER(WsCounts)]
+    L.ws_loopmerge_unrolled(_p(nsteps, C.c_uint32), _p(ev_flat, C.c_uint16),
+                            _p(ev_off, C.c_uint64), W, n_valid, K, mode, T, U, C.byref(o))
     return o.as_dict(LM)
 
 

@@ -165,6 +165,10 @@ void ws_commoncall(const uint8_t* arm, uint32_t W, uint32_t n_valid, int mode, w
 /* Loop merge: lane l owns tasks k < K; task (l,k) runs nsteps[l*K+k] >= 1 inner
  * iterations; ev (may be NULL) gives each step's bit0 = boundary, laid out
  * per task at ev_off[l*K+k]. */
+/* Loop Merge with the merged inner loop partially unrolled by U (U = 1: plain) */
+void ws_loopmerge_unrolled(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
+                           uint32_t W, uint32_t n_valid, uint32_t K, int mode, uint32_t T,
+                           uint32_t U, ws_counts* out);
 /* Loop Merge + nested Iteration Delay of the boundary sub-step (warpsim.c) */
 void ws_loopmerge_defer(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
                         uint32_t W, uint32_t n_valid, uint32_t K, uint32_t T, uint32_t Tb,

@@ -139,6 +139,16 @@ static void step_split(ws_counts* o, const or_event* ev, const uint64_t* ev_off,
 
 void ws_loopmerge(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off, uint32_t W,
                   uint32_t n_valid, uint32_t K, int mode, uint32_t T, ws_counts* o) {
+  ws_loopmerge_unrolled(nsteps, ev, ev_off, W, n_valid, K, mode, T, 1, o);
+}
+
+/* U > 1: the merged inner loop partially unrolled by U: a
+ * release runs up to U steps; a lane whose task ends inside the release idles
+ * for the rest of it ("reconvergence is needed only once per N iterations"). */
+void ws_loopmerge_unrolled(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
+                           uint32_t W, uint32_t n_valid, uint32_t K, int mode, uint32_t T,
+                           uint32_t U, ws_counts* o) {
+  if (U == 0) U = 1;
   memset(o, 0, sizeof *o);
   if (n_valid > W) n_valid = W;
   uint32_t valid = n_valid >= 32 ? 0xffffffffu : ((1u << n_valid) - 1u);
@@ -175,14 +185,17 @@ void ws_loopmerge(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev
     hit(o, WS_LM_ROUND, valid);
     if ((uint32_t)__builtin_popcount(P) >= T || !R) {
       hit(o, WS_LM_RELEASE, P);
-      hit(o, WS_LM_STEP, P);
-      if (ev) {
-        step_split(o, ev, ev_off, K, kk, jj, P);
-      }
-      for (uint32_t l = 0; l < n_valid; ++l) {
-        if (!(P >> l & 1u)) continue;
-        jj[l] += 1;
-        if (jj[l] == nsteps[l * K + kk[l]]) alive &= ~(1u << l);
+      uint32_t S = P;
+      for (uint32_t r = 0; r < U && S; ++r) {
+        hit(o, WS_LM_STEP, S);
+        if (ev) {
+          step_split(o, ev, ev_off, K, kk, jj, S);
+        }
+        for (uint32_t l = 0; l < n_valid; ++l) {
+          if (!(S >> l & 1u)) continue;
+          jj[l] += 1;
+          if (jj[l] == nsteps[l * K + kk[l]]) { alive &= ~(1u << l); S &= ~(1u << l); }
+        }
       }
     } else {
       hit(o, WS_LM_ADVANCE, R);

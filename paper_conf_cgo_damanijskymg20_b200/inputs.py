@@ -66,6 +66,7 @@ class MCML:
     n_threads: int = 156250     # lanes
     iters: int = 64             # photons per lane (thread coarsening)
     threshold: int = 32
+    merge_unroll: int = 4       # photon steps per release, tuned on B200
 
     @property
     def n_photons(self) -> int:

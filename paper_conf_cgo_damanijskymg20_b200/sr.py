@@ -54,7 +54,8 @@ class CommoncallParams(C.Structure):
 class MCMLParams(C.Structure):
     _fields_ = [("n_layers", C.c_uint32), ("layers", Layer * MAX_LAYERS), ("n_above", C.c_float),
                 ("n_below", C.c_float), ("dr", C.c_float), ("dz", C.c_float), ("nr", C.c_uint32),
-                ("nz", C.c_uint32), ("step_cap", C.c_uint32), ("defer_threshold", C.c_uint32)]
+                ("nz", C.c_uint32), ("step_cap", C.c_uint32), ("defer_threshold", C.c_uint32),
+                ("merge_unroll", C.c_uint32)]
 
 
 class PathtraceParams(C.Structure):
@@ -205,7 +206,7 @@ def commoncall_workload(fma_count=2000, split_u32=1 << 31, task_offset=0, flags=
 
 def mcml_workload(layers, n_above=1.0, n_below=1.0, dr=0.01, dz=0.002, nr=256, nz=255,
                   step_cap=100000, task_offset=0, flags=0, block=0, grid=0,
-                  defer=0) -> Workload:
+                  defer=0, unroll=0) -> Workload:
     w = Workload(kind=WL_MCML, flags=flags, task_offset=task_offset, block_threads=block,
                  grid_ctas=grid)
     m = MCMLParams()
@@ -215,6 +216,7 @@ def mcml_workload(layers, n_above=1.0, n_below=1.0, dr=0.01, dz=0.002, nr=256, n
     m.n_above, m.n_below, m.dr, m.dz = n_above, n_below, dr, dz
     m.nr, m.nz, m.step_cap = nr, nz, step_cap
     m.defer_threshold = defer
+    m.merge_unroll = unroll
     w.mcml = m
     return w
 

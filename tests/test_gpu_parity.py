@@ -238,6 +238,35 @@ def test_mcml_schedule_matches_simulator(ctx, mode, T):
 
 
 @pytest.mark.parametrize("flags", [0, sr.F_STATIC])
+@pytest.mark.parametrize("T,U", [(32, 2), (32, 4), (16, 3)])
+def test_mcml_unrolled_merge_bit_exact(ctx, flags, T, U):
+    m = I.C3
+    nt, it = 300, 5
+    ref = mc_oracle(m, 0, nt * it, 19)
+    got = run_mc(ctx, mc_workload(m, flags=flags, block=128, unroll=U), nt, it, 19,
+                 sr.SPEC_LOOP, T, m)
+    assert_mc_equal(got, ref)
+
+
+@pytest.mark.parametrize("T,U", [(32, 2), (8, 4)])
+def test_mcml_unrolled_schedule_matches_simulator(ctx, T, U):
+    m = I.C3
+    nt, it = 96, 6
+    w = mc_workload(m, flags=sr.F_STATIC | sr.F_SCHED, block=32, unroll=U)
+    run_mc(ctx, w, nt, it, 3, sr.SPEC_LOOP, T, m)
+    sched = ctx.region(w, nt, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    p = oracle.mc_params(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap)
+    ev, off, ns = oracle.mcml_events_batch(p, 0, nt * it, 3)
+    for wi in range(nt // 32):
+        lanes = np.arange(32 * wi, 32 * wi + 32)
+        ids = lanes[:, None] + np.arange(it)[None, :] * nt
+        s = oracle.ws_loopmerge_raw(ns[ids], ev, off[ids].ravel(), oracle.SPEC_LOOP, T, U=U)
+        g = sched[wi]
+        assert g[0] == s["rounds"] and (g[1], g[2]) == s["RELEASE"], wi
+        assert (g[3], g[4]) == s["LAUNCH"], wi
+
+
+@pytest.mark.parametrize("flags", [0, sr.F_STATIC])
 @pytest.mark.parametrize("T,Tb", [(32, 1), (32, 8), (16, 4), (32, 32)])
 def test_mcml_deferred_boundary_bit_exact(ctx, flags, T, Tb):
     m = I.C3

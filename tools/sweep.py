@@ -69,7 +69,7 @@ if "mcml" in a.what:
     res = []
     for b in blocks:
         w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
-                             block=b, defer=a.defer)
+                             block=b, defer=a.defer, unroll=a.unroll)
         ctx.ensure(sr.sr_workspace_bytes(w, nt))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
             t = timed(lambda: sr.sr_run(w, nt, m.iters, seed, mode, T), a.reps)
