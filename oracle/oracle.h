@@ -146,9 +146,10 @@ enum { WS_LM_ENTRY = 0, WS_LM_LAUNCH, WS_LM_STEP, WS_LM_STEP_BOUNDARY,
        WS_LM_STEP_INTERACT, WS_LM_ROUND, WS_LM_RELEASE, WS_LM_ADVANCE,
        WS_LM_EV0 = 8,      /* .. WS_LM_EV0+15: step lanes whose event has bit b set   */
        WS_LM_NEV0 = 24,    /* .. WS_LM_NEV0+15: step lanes whose event has bit b clear */
-       WS_LM_A_RR = 40,    /* deferred mode: roulette of interaction steps (part A)   */
-       WS_LM_B_RR = 41,    /* deferred mode: roulette of boundary steps (part B)      */
-       WS_LM_B_REL = 42,   /* deferred mode: boundary releases, lanes = parked set    */
+       WS_LM_A_RR = 40,    /* roulette of interaction steps (part A)                  */
+       WS_LM_B_RR = 41,    /* roulette of boundary steps (part B)                     */
+       WS_LM_B_REL = 42,   /* part B of a boundary step; deferred mode: the release,
+                              lanes = parked set                                      */
        WS_LM_NREG = 43 };
 #define WS_MAX_REG 48
 typedef struct {

@@ -131,6 +131,11 @@ static void step_split(ws_counts* o, const or_event* ev, const uint64_t* ev_off,
   }
   hit(o, WS_LM_STEP_BOUNDARY, set[0]);
   hit(o, WS_LM_STEP_INTERACT, mask & ~set[0]);
+  /* the same step written as part A + part B (boundary lanes) with each part's
+   * roulette: the regions ws_loopmerge_defer costs separately */
+  hit(o, WS_LM_B_REL, set[0]);
+  hit(o, WS_LM_A_RR, set[5] & ~set[0]);
+  hit(o, WS_LM_B_RR, set[5] & set[0]);
   for (int b = 0; b < 16; ++b) {
     hit(o, WS_LM_EV0 + b, set[b]);
     hit(o, WS_LM_NEV0 + b, mask & ~set[b]);

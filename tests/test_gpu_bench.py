@@ -43,12 +43,12 @@ def test_bench_two_rank_path_gloo():
     r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
                         "--nproc-per-node", "2", "--master-addr", "127.0.0.1", "--master-port",
                         "29541", "bench.py", "--gpus", "2", "--steps", "3", "--warmup", "3",
-                        "--dist-backend", "gloo", "--photons-per-gpu", "500000"],
+                        "--dist-backend", "gloo", "--photons-per-gpu", "512000"],
                        cwd=ROOT, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stderr[-2000:]
     d = _last_json(r.stdout)
     assert d["n_gpus"] == 2 and d["scaling"] == "weak"
-    assert d["config"]["photons_per_gpu"] == 500000
+    assert d["config"]["photons_per_gpu"] == 512000   # a multiple of photons_per_lane
     assert "cpu_baseline" not in d and "configs" not in d   # rank 0 at N=1 only
 
 

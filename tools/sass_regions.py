@@ -59,15 +59,26 @@ def marked_call_lines(path):
     (e.g. the MC step): an instruction resolved only to such a line lost its
     intermediate inline frames."""
     src = open(path).read().splitlines()
-    fn, marked = None, set()
+    fn, marked, body = None, set(), {}
     for line in src:
         m = re.search(r"__device__[^(;]*?\b(\w+)\s*\(", line)
         if m and "__global__" not in line:
             fn = m.group(1)
         elif "__global__" in line:
             fn = None
-        if fn and MARK_RE.search(line):
-            marked.add(fn)
+        if fn:
+            body.setdefault(fn, []).append(line.split("//")[0])
+            if MARK_RE.search(line):
+                marked.add(fn)
+    # transitively: a function calling a marked function (MC step -> step_a/b)
+    changed = True
+    while changed:
+        changed = False
+        for f, lines in body.items():
+            if f not in marked and any(re.search(r"\b%s\s*\(" % g, c)
+                                       for g in marked for c in lines[1:]):
+                marked.add(f)
+                changed = True
     out = set()
     for i, line in enumerate(src, 1):
         code = line.split("//")[0]
