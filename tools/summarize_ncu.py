@@ -76,6 +76,8 @@ def row_of(kname, m):
                 dram_bytes=(num(m.get("dram__bytes_read.sum")) or 0) +
                 (num(m.get("dram__bytes_write.sum")) or 0),
                 l2_bytes=num(m.get("lts__t_bytes.sum")),
+                ffma_thread_inst=num(m.get("sm__sass_thread_inst_executed_op_ffma_pred_on.sum")),
+                ffma2_thread_inst=num(m.get("sm__sass_thread_inst_executed_op_ffma2_pred_on.sum")),
                 regs=num(m.get("launch__registers_per_thread")),
                 grid=num(m.get("launch__grid_size")), block=num(m.get("launch__block_size")))
 

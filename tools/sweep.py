@@ -26,6 +26,8 @@ ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--flags", type=int, default=0, help="extra sr_workload.flags (e.g. 4 = F_COARSE)")
 ap.add_argument("--unroll", type=int, default=0, help="PT node-merge partial unroll")
 ap.add_argument("--defer", type=int, default=0, help="MCML boundary defer threshold T_b")
+ap.add_argument("--static", action="store_true", help="MCML static photon assignment (F_STATIC)")
+ap.add_argument("--iters", type=int, default=0, help="MCML photons per lane (default configs[2])")
 a = ap.parse_args()
 Ts = [int(x) for x in a.thresholds.split(",")]
 blocks = [int(x) for x in a.blocks.split(",")]
@@ -65,17 +67,20 @@ def eff(w, n, iters, mode, T):
 out = {}
 if "mcml" in a.what:
     m = I.C3
-    nt = a.photons // m.iters
+    iters = a.iters or m.iters
+    nt = a.photons // iters
     res = []
     for b in blocks:
         w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
-                             block=b, defer=a.defer, unroll=a.unroll)
+                             block=b, defer=a.defer, unroll=a.unroll,
+                             flags=sr.F_STATIC if a.static else 0)
         ctx.ensure(sr.sr_workspace_bytes(w, nt))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
-            t = timed(lambda: sr.sr_run(w, nt, m.iters, seed, mode, T), a.reps)
+            t = timed(lambda: sr.sr_run(w, nt, iters, seed, mode, T), a.reps)
             r = dict(block=b, mode="pdom" if mode == sr.PDOM else "spec", T=T, ms=t,
-                     photons_per_s=nt * m.iters / (t * 1e-3), launch=sr.sr_last_launch())
-            r.update(eff(w, min(nt, 65536), m.iters, mode, T))
+                     photons_per_s=nt * iters / (t * 1e-3), launch=sr.sr_last_launch(),
+                     unroll=a.unroll, static=a.static, photons=nt * iters)
+            r.update(eff(w, min(nt, 65536), iters, mode, T))
             res.append(r)
             print(json.dumps(r), file=sys.stderr, flush=True)
     out["mcml"] = res
