@@ -68,6 +68,13 @@ typedef enum {
 #define SR_F_COARSE 4u  /* PATHTRACE + SR_SPEC_LOOP: merge at bounce granularity (one release =
                            traversal + shading of one bounce) instead of the default BVH-node
                            granularity (one release = one node visit). Results are identical. */
+#define SR_F_NOSPLIT 8u /* PATHTRACE + SR_SPEC_LOOP at node granularity: one merged region per
+                           node visit (its leaf triangle tests inline) instead of the default
+                           two concurrent predictions, where inner-node visits
+                           and leaf triangle tests are separate regions and each round runs the
+                           larger waiting group (soft barrier T) while the other lanes wait.
+                           Results and counters are identical (each lane's traversal order is
+                           the same). */
 
 #define SR_MAX_LAYERS 8
 typedef struct { float n, mua, mus, g, d; } sr_layer;  /* -, 1/cm, 1/cm, -, cm */

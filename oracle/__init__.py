@@ -31,10 +31,10 @@ DL = dict(ENTRY=0, PROLOG=1, EXPENSIVE=2, EPILOG=3, ROUND=4, RELEASE=5, ADVANCE=
 CC = dict(ENTRY=0, THEN=1, ELSE_PRE=2, CALL=3, ELSE_POST=4, MERGE=5)
 LM = dict(ENTRY=0, LAUNCH=1, STEP=2, STEP_BOUNDARY=3, STEP_INTERACT=4, ROUND=5, RELEASE=6,
           ADVANCE=7, **{f"EV{b}": 8 + b for b in range(16)}, **{f"NEV{b}": 24 + b for b in range(16)},
-          A_RR=40, B_RR=41, B_REL=42)
+          A_RR=40, B_RR=41, B_REL=42, BI=43, A_TAIL=44)
 # MC step event bits (oracle.h OR_EV_*)
 EV_BOUNDARY, EV_SLEFT, EV_REFLECT, EV_EXIT, EV_TRANSMIT, EV_ROULETTE, EV_SPIN_AXIS, \
-    EV_SPIN_GENERAL, EV_EXTERNAL = 1, 2, 4, 8, 16, 32, 64, 128, 256
+    EV_SPIN_GENERAL, EV_EXTERNAL, EV_MATCHED = 1, 2, 4, 8, 16, 32, 64, 128, 256, 512
 MC_COUNTERS = ["photons", "steps", "rd_exits", "tt_exits", "rr_kills", "rr_survive", "capped",
                "zero_w"]
 MAX_LAYERS = 8

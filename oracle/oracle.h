@@ -91,7 +91,8 @@ void or_mcml(const or_mcml_params* p, uint64_t id0, uint64_t count, uint64_t see
 typedef uint16_t or_event;
 enum { OR_EV_BOUNDARY = 1, OR_EV_SLEFT = 2, OR_EV_REFLECT = 4, OR_EV_EXIT = 8,
        OR_EV_TRANSMIT = 16, OR_EV_ROULETTE = 32, OR_EV_SPIN_AXIS = 64,
-       OR_EV_SPIN_GENERAL = 128, OR_EV_EXTERNAL = 256 /* boundary with the ambient */ };
+       OR_EV_SPIN_GENERAL = 128, OR_EV_EXTERNAL = 256 /* boundary with the ambient */,
+       OR_EV_MATCHED = 512 /* boundary with a layer of equal index: Fresnel r = 0 */ };
 uint32_t or_mcml_events(const or_mcml_params* p, uint64_t id, uint64_t seed,
                         or_event* ev, uint32_t cap);
 uint64_t or_mcml_events_batch(const or_mcml_params* p, uint64_t id0, uint64_t count,
@@ -150,7 +151,9 @@ enum { WS_LM_ENTRY = 0, WS_LM_LAUNCH, WS_LM_STEP, WS_LM_STEP_BOUNDARY,
        WS_LM_B_RR = 41,    /* roulette of boundary steps (part B)                     */
        WS_LM_B_REL = 42,   /* part B of a boundary step; deferred mode: the release,
                               lanes = parked set                                      */
-       WS_LM_NREG = 43 };
+       WS_LM_BI = 43,      /* matched boundary finished inside part A (no part B)     */
+       WS_LM_A_TAIL = 44,  /* end of part A: interaction + matched-boundary lanes     */
+       WS_LM_NREG = 45 };
 #define WS_MAX_REG 48
 typedef struct {
   uint64_t rounds;                 /* SR scheduler rounds (0 under PDOM) */

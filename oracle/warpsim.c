@@ -131,11 +131,21 @@ static void step_split(ws_counts* o, const or_event* ev, const uint64_t* ev_off,
   }
   hit(o, WS_LM_STEP_BOUNDARY, set[0]);
   hit(o, WS_LM_STEP_INTERACT, mask & ~set[0]);
-  /* the same step written as part A + part B (boundary lanes) with each part's
-   * roulette: the regions ws_loopmerge_defer costs separately */
-  hit(o, WS_LM_B_REL, set[0]);
-  hit(o, WS_LM_A_RR, set[5] & ~set[0]);
-  hit(o, WS_LM_B_RR, set[5] & set[0]);
+  /* the same step written as part A + part B with each part's roulette (the
+   * regions ws_loopmerge_defer costs separately): a boundary with a layer of
+   * equal index (bit 9) is finished inside part A; the other boundary lanes
+   * run part B */
+  const uint32_t b_lanes = set[0] & ~set[9];
+  hit(o, WS_LM_BI, set[9]);
+  hit(o, WS_LM_A_TAIL, mask & ~b_lanes);
+  hit(o, WS_LM_A_RR, set[5] & ~b_lanes);
+  hit(o, WS_LM_B_REL, b_lanes);
+  hit(o, WS_LM_B_RR, set[5] & b_lanes);
+  /* reflect / exit / transmit (bits 2-4) are branches of part B: a matched
+   * boundary's reflect or transmit runs inside part A (BI) instead */
+  set[2] &= b_lanes;
+  set[3] &= b_lanes;
+  set[4] &= b_lanes;
   for (int b = 0; b < 16; ++b) {
     hit(o, WS_LM_EV0 + b, set[b]);
     hit(o, WS_LM_NEV0 + b, mask & ~set[b]);
@@ -226,7 +236,8 @@ void ws_loopmerge_unrolled(const uint32_t* nsteps, const or_event* ev, const uin
  *   |B| >= Tb -> boundary release; else |P| >= T -> step release;
  *   else R != {} -> advance; else P != {} -> step release; else B != {} ->
  *   boundary release; else exit.
- * Only the boundary bit (bit0) of the events decides the schedule; the other
+ * Only the boundary bits (bit0, and bit9: a matched boundary finishes in part
+ * A and does not park) of the events decide the schedule; the other
  * bits split each phase's mask for costing: phase A counts bits 1, 6, 7 and
  * the interaction roulette; phase B counts bits 2, 3, 4, 8 and its roulette. */
 static or_event evt(const or_event* ev, const uint64_t* ev_off, uint32_t K, const uint32_t* kk,
@@ -274,10 +285,13 @@ void ws_loopmerge_defer(const uint32_t* nsteps, const or_event* ev, const uint64
       hit(o, WS_LM_NEV0 + 1, P & ~bit[1]);
       hit(o, WS_LM_EV0 + 6, bit[6]);
       hit(o, WS_LM_EV0 + 7, bit[7]);
-      hit(o, WS_LM_A_RR, bit[5] & ~bit[0]);
+      const uint32_t b_lanes = bit[0] & ~bit[9];   /* matched boundaries finish in A */
+      hit(o, WS_LM_BI, bit[9]);
+      hit(o, WS_LM_A_TAIL, P & ~b_lanes);
+      hit(o, WS_LM_A_RR, bit[5] & ~b_lanes);
       for (uint32_t l = 0; l < n_valid; ++l) {
         if (!(P >> l & 1u)) continue;
-        if (bit[0] >> l & 1u) { parked |= 1u << l; continue; }   /* Join + Wait */
+        if (b_lanes >> l & 1u) { parked |= 1u << l; continue; }   /* Join + Wait */
         jj[l] += 1;
         if (jj[l] == nsteps[l * K + kk[l]]) alive &= ~(1u << l);
       }

@@ -257,8 +257,27 @@ extern "C" int sr_scene_build(const float* tris, const uint32_t* mat, uint32_t n
     }
   }
 
+  // traversal stack bound: a visit pushes at most one entry (the farther of
+  // two inner children), so a ray holds at most (inner nodes on its root path
+  // - 1) entries
+  uint32_t stack_need = 0;
+  {
+    std::vector<std::pair<int, uint32_t>> st{{0, 0u}};
+    while (!st.empty()) {
+      const auto [i, d] = st.back();
+      st.pop_back();
+      stack_need = std::max(stack_need, d);
+      const PtNode& o = nodes[i];
+      const bool in0 = o.ref0 >= 0 && o.cnt0 == 0, in1 = o.ref1 >= 0 && o.cnt1 == 0;
+      const uint32_t dd = d + ((in0 && in1) ? 1u : 0u);
+      if (in0) st.push_back({o.ref0, dd});
+      if (in1) st.push_back({o.ref1, dd});
+    }
+  }
+
   std::vector<unsigned char> img(bound, 0);
   PtHeader h{};
+  h.stack_need = stack_need;
   h.magic = kPtMagic;
   h.n_nodes = (uint32_t)nodes.size();
   h.n_tris = n_tris;

@@ -11,11 +11,18 @@
 //
 //   pt_pdom  as written: a warp's 32 pixels trace sample s together; lanes
 //            whose path ended idle until the longest path of the warp ends.
-//   pt_spec  Loop Merge + soft barrier: P = ballot(path in flight); if
-//            popc(P) >= T or no idle lane has a sample left, every in-flight
-//            lane takes one bounce; otherwise idle lanes run the epilog and
-//            the next camera ray.  "PathTracer executes fastest when all
-//            threads reconverge" -> default T = 32.
+//   pt_spec  Loop Merge + soft barrier at one of three granularities:
+//            bounce (SR_F_COARSE): P = ballot(path in flight); if popc(P) >= T
+//              or no idle lane has a sample left, every in-flight lane takes
+//              one bounce; otherwise idle lanes run the epilog and the next
+//              camera ray;
+//            node (SR_F_NOSPLIT): the same one nesting level deeper, one
+//              release = merge_unroll BVH node visits;
+//            split (default): two concurrent predictions --
+//              lanes at an inner node and lanes with leaf triangles pending
+//              are separate candidate sets; each round releases the larger
+//              (soft barrier T), the other waits (Iteration Delay's vote,
+//              P:1552-1557).
 //
 // One lane = one pixel (static; the pixel sum is accumulated in sample order,
 // so the float result is schedule-free).  bounce() = BVH closest hit (exactly
@@ -31,7 +38,19 @@ namespace {
 
 constexpr float kTmin = 1.0e-4f;
 constexpr float kDetEps = 1.0e-12f;
-constexpr int kStack = 64;  // > BVH depth (binned SAH over 1M triangles: ~40)
+// traversal stack: one column of PtHeader.stack_need entries per thread in
+// dynamic shared memory (23 for configs[3]); kMaxStack bounds what a scene may need
+constexpr uint32_t kMaxStack = 256;
+// CTAs of 128 threads per SM the register budget must allow, per kernel, each
+// at its best measured setting (profiles/pt_tuning_r01.md): the latency-bound
+// PDOM kernel wants 8 (64 registers), the merged kernels 6 (80 registers).
+// (An L1 prefetch of the next node / triangle was measured 5 % slower.)
+#ifndef SR_PT_MINB_PDOM
+#define SR_PT_MINB_PDOM 8
+#endif
+#ifndef SR_PT_MINB_SPEC
+#define SR_PT_MINB_SPEC 6
+#endif
 
 struct V3 {
   float x, y, z;
@@ -56,6 +75,7 @@ struct PtArgs {
   const PtMat* mats;
   uint32_t width, height, spp, max_depth, T;
   uint32_t unroll;                  // node visits per release (partial unroll)
+  uint32_t stack_cap;               // traversal stack entries per thread (>= stack_need)
   uint64_t n, seed;
   RoundKeys keys;
   float* rgb;                       // 3 floats per pixel
@@ -129,6 +149,10 @@ struct Trav {
   int32_t sp;
   int32_t* stk;     // this thread's column of the CTA's shared stack
   uint32_t stride;  // blockDim.x
+  // split merge (default): leaf ranges found by the last node visit, tested later by
+  // trav_leaf (current range la/na, queued range lb/nb)
+  int32_t la, lb;
+  uint32_t na, nb;
 };
 
 __device__ __forceinline__ void trav_bind(Trav& tr) {
@@ -147,6 +171,8 @@ __device__ __forceinline__ void trav_begin(Trav& tr, V3 o, V3 d) {
   tr.slot = 0;
   tr.node = 0;
   tr.sp = 0;
+  tr.na = 0;
+  tr.nb = 0;
 }
 
 // returns false when the traversal is finished
@@ -178,7 +204,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
   if (in0 && in1) {
     const bool first0 = tn0 <= tn1;
     next = first0 ? N.ref0 : N.ref1;
-    if (tr.sp < kStack) tr.stk[(tr.sp++) * tr.stride] = first0 ? N.ref1 : N.ref0;
+    if ((uint32_t)tr.sp < a.stack_cap) tr.stk[(tr.sp++) * tr.stride] = first0 ? N.ref1 : N.ref0;
   } else if (in0) {
     next = N.ref0;
   } else if (in1) {
@@ -190,6 +216,51 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
   }
   tr.node = next;
   return true;
+}
+
+// Split merge (default): trav_step cut into its two regions, each lane's sequence of
+// node visits and triangle tests unchanged.  trav_node visits tr.node: box
+// tests, queues the hit leaf children (child 0 first) for trav_leaf, picks
+// the next node exactly as trav_step (node = -1 when the stack is empty).
+// trav_leaf tests ONE queued triangle.  Returns: a leaf triangle is pending
+// (na > 0), else a node is pending (node >= 0), else the traversal is done.
+__device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, Stats& st) {
+  const PtNode N = a.nodes[tr.node];
+  ++st.nodes;
+  float tn0, tn1;
+  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, tr.o, tr.inv, tr.tb, tn0);
+  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, tr.o, tr.inv, tr.tb, tn1);
+  const bool l0 = h0 && N.cnt0 > 0, l1 = h1 && N.cnt1 > 0;
+  tr.la = l0 ? N.ref0 : N.ref1;
+  tr.na = l0 ? (uint32_t)N.cnt0 : (l1 ? (uint32_t)N.cnt1 : 0u);
+  tr.lb = N.ref1;
+  tr.nb = (l0 && l1) ? (uint32_t)N.cnt1 : 0u;
+  const bool in0 = h0 && N.cnt0 == 0, in1 = h1 && N.cnt1 == 0;
+  int32_t next = -1;
+  if (in0 && in1) {
+    const bool first0 = tn0 <= tn1;
+    next = first0 ? N.ref0 : N.ref1;
+    if ((uint32_t)tr.sp < a.stack_cap) tr.stk[(tr.sp++) * tr.stride] = first0 ? N.ref1 : N.ref0;
+  } else if (in0) {
+    next = N.ref0;
+  } else if (in1) {
+    next = N.ref1;
+  }
+  if (next < 0 && tr.sp > 0) next = tr.stk[(--tr.sp) * tr.stride];
+  tr.node = next;
+}
+
+__device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, Stats& st) {
+  const int64_t before = tr.ib;
+  tri_test(a.tris[tr.la], tr.o, tr.d, tr.tb, tr.ib, tr.mb);
+  if (tr.ib != before) tr.slot = (uint32_t)tr.la;
+  ++st.tests;
+  ++tr.la;
+  if (--tr.na == 0u) {
+    tr.la = tr.lb;
+    tr.na = tr.nb;
+    tr.nb = 0u;
+  }
 }
 
 __device__ __forceinline__ int64_t closest_hit(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
@@ -303,7 +374,8 @@ __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
 __device__ __forceinline__ void finish(const PtArgs& a, const Path& p, bool valid, Stats st,
                                        uint32_t paths, uint64_t warp, uint32_t rounds,
                                        uint32_t rel, uint32_t rel_lanes, uint32_t adv,
-                                       uint32_t adv_lanes) {
+                                       uint32_t adv_lanes, uint32_t lrel = 0,
+                                       uint32_t lrel_lanes = 0) {
   if (valid) {
     a.rgb[3 * (uint64_t)p.pix + 0] = p.sum.x;
     a.rgb[3 * (uint64_t)p.pix + 1] = p.sum.y;
@@ -321,7 +393,7 @@ __device__ __forceinline__ void finish(const PtArgs& a, const Path& p, bool vali
     if (a.sched) {
       uint4* s = reinterpret_cast<uint4*>(a.sched + warp * kSchedWords);
       s[0] = make_uint4(rounds, rel, rel_lanes, adv);
-      s[1] = make_uint4(adv_lanes, 0u, 0u, 0u);
+      s[1] = make_uint4(adv_lanes, lrel, lrel_lanes, 0u);
     }
   }
 }
@@ -333,7 +405,7 @@ __device__ __forceinline__ void bounce(const PtArgs& a, Path& p, Trav& tr, Stats
 }
 
 template <bool SCHED>
-__global__ void __launch_bounds__(128) pt_pdom(const PtArgs a) {
+__global__ void __launch_bounds__(128, SR_PT_MINB_PDOM) pt_pdom(const PtArgs a) {
   const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = g < a.n;
@@ -371,9 +443,10 @@ __global__ void __launch_bounds__(128) pt_pdom(const PtArgs a) {
 // every lane with a ray in flight); shading, the pixel epilog and the next
 // camera ray form the advance step.  The second is Loop Merge applied one
 // nesting level deeper (P:1514-1528 leaves nesting open), where the trip
-// count (nodes per ray) varies most.
-template <bool SCHED, bool NODE>
-__global__ void __launch_bounds__(128) pt_spec(const PtArgs a) {
+// count (nodes per ray) varies most.  SPLIT (with NODE): the node visit's
+// leaf triangle tests become their own region (trav_node / trav_leaf).
+template <bool SCHED, bool NODE, bool SPLIT = false>
+__global__ void __launch_bounds__(128, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) {
   const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = g < a.n;
@@ -389,7 +462,51 @@ __global__ void __launch_bounds__(128) pt_spec(const PtArgs a) {
   uint32_t paths = 0, rounds = 0, rel = 0, rel_lanes = 0, adv = 0, adv_lanes = 0;
   uint32_t next_s = 0;
   uint32_t E = __ballot_sync(kFull, !valid || a.spp == 0);  // lanes with nothing left to do
+  uint32_t lrel = 0, lrel_lanes = 0;
   for (;;) {
+    if constexpr (SPLIT) {
+      // two concurrent predictions: I = lanes at a BVH node, L = lanes with a
+      // leaf triangle pending.  Vote: the larger group G is the candidate
+      // release (soft barrier T); the other group waits (Iteration Delay).
+      const uint32_t L = __ballot_sync(kFull, trav && tr.na > 0u);
+      const uint32_t I = __ballot_sync(kFull, trav && tr.na == 0u);
+      const uint32_t R = ~(I | L | E);
+      if ((I | L | R) == 0u) break;
+      if constexpr (SCHED) ++rounds;
+      const bool leaf = __popc(L) > __popc(I);
+      const uint32_t G = leaf ? L : I;
+      if (G != 0u && ((uint32_t)__popc(G) >= a.T || R == 0u)) {
+        if ((G >> lane_id()) & 1u) {
+          __syncwarp(G);
+          if (leaf) {
+            if constexpr (SCHED) { ++lrel; lrel_lanes += __popc(G); }
+            for (uint32_t k = 0; k < a.unroll && tr.na > 0u; ++k) trav_leaf(a, tr, st);
+          } else {
+            if constexpr (SCHED) { ++rel; rel_lanes += __popc(G); }
+            for (uint32_t k = 0; k < a.unroll && tr.na == 0u && tr.node >= 0; ++k)
+              trav_node(a, tr, st);
+          }
+          trav = tr.na > 0u || tr.node >= 0;
+        }
+        continue;
+      }
+      if constexpr (SCHED) { ++adv; adv_lanes += __popc(R); }
+      if ((R >> lane_id()) & 1u) {
+        if (p.alive) shade(a, p, tr);
+        if (!p.alive && next_s < a.spp) {
+          p.s = next_s++;
+          camera_ray(a, H, p);
+          ++paths;
+        }
+        if (p.alive) {
+          trav_begin(tr, p.o, p.d);
+          ++st.rays;
+          trav = true;
+        }
+      }
+      E = __ballot_sync(kFull, !valid || (!p.alive && next_s >= a.spp));
+      continue;
+    }
     const uint32_t P = __ballot_sync(kFull, NODE ? trav : p.alive);
     const uint32_t R = ~(P | E);
     if ((P | R) == 0u) break;
@@ -421,7 +538,8 @@ __global__ void __launch_bounds__(128) pt_spec(const PtArgs a) {
       E = __ballot_sync(kFull, !valid || (!p.alive && next_s >= a.spp));
     }
   }
-  finish(a, p, valid, st, paths, g >> 5, rounds, rel, rel_lanes, adv, adv_lanes);
+  finish(a, p, valid, st, paths, g >> 5, rounds, rel, rel_lanes, adv, adv_lanes, lrel,
+         lrel_lanes);
 }
 
 // sr_pt_closest diagnostics: one ray per thread
@@ -481,6 +599,8 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
   a.spp = iters;
   a.max_depth = w.pathtrace.max_depth;
   a.unroll = w.pathtrace.merge_unroll ? w.pathtrace.merge_unroll : 8;
+  if (h.stack_need > kMaxStack) return cudaErrorInvalidValue;
+  a.stack_cap = h.stack_need > 0 ? h.stack_need : 1u;
   a.T = T;
   a.n = n;
   a.seed = seed;
@@ -495,7 +615,7 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
   const bool spec = mode == SR_SPEC_LOOP;
   const bool node = (w.flags & SR_F_COARSE) == 0;
   const unsigned gr = (unsigned)grid;
-  const size_t smem = (size_t)kStack * block * sizeof(int32_t);  // traversal stacks
+  const size_t smem = (size_t)a.stack_cap * block * sizeof(int32_t);  // traversal stacks
   if (smem > 227 * 1024) return cudaErrorInvalidConfiguration;
   record_launch((uint32_t)grid, block, (uint32_t)smem);
   if (smem > 48 * 1024) {
@@ -505,10 +625,15 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
     cudaFuncSetAttribute(pt_spec<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaFuncSetAttribute(pt_spec<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaFuncSetAttribute(pt_spec<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<false, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<true, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   }
   if (!spec) {
     if (a.sched) pt_pdom<true><<<gr, block, smem, c.stream>>>(a);
     else pt_pdom<false><<<gr, block, smem, c.stream>>>(a);
+  } else if (node && !(w.flags & SR_F_NOSPLIT)) {
+    if (a.sched) pt_spec<true, true, true><<<gr, block, smem, c.stream>>>(a);
+    else pt_spec<false, true, true><<<gr, block, smem, c.stream>>>(a);
   } else if (node) {
     if (a.sched) pt_spec<true, true><<<gr, block, smem, c.stream>>>(a);
     else pt_spec<false, true><<<gr, block, smem, c.stream>>>(a);
@@ -532,9 +657,11 @@ cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* ray
   a.q_rays = rays;
   a.q_hit = hit;
   a.q_t = t;
+  if (h.stack_need > kMaxStack) return cudaErrorInvalidValue;
+  a.stack_cap = h.stack_need > 0 ? h.stack_need : 1u;
   const unsigned grid = (unsigned)((n + 127) / 128);
   record_launch(grid, 128, 0);
-  if (n) pt_query<<<grid, 128, kStack * 128 * sizeof(int32_t), st>>>(a);
+  if (n) pt_query<<<grid, 128, a.stack_cap * 128 * sizeof(int32_t), st>>>(a);
   return cudaGetLastError();
 }
 

@@ -21,7 +21,8 @@ struct PtHeader {
   uint32_t magic, n_nodes, n_tris, n_mats;
   uint64_t off_nodes, off_tris, off_mats, bytes;
   float cam[16];      // eye, forward, right, up, tan(fov/2), aspect
-  uint32_t pad[4];
+  uint32_t stack_need;  // deepest traversal stack any ray can need (entries)
+  uint32_t pad[3];
 };
 static_assert(sizeof(PtHeader) == 128, "PtHeader layout");
 

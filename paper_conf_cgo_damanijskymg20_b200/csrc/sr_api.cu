@@ -48,7 +48,7 @@ std::string check_workload(const sr_workload* w, uint64_t n_threads) {
   if (w->block_threads != 0 &&
       (w->block_threads % 32 != 0 || w->block_threads < 32 || w->block_threads > 1024))
     return "block_threads must be 0 or a multiple of 32 in [32, 1024]";
-  if (w->flags & ~(SR_F_SCHED | SR_F_STATIC | SR_F_COARSE)) return "unknown flags";
+  if (w->flags & ~(SR_F_SCHED | SR_F_STATIC | SR_F_COARSE | SR_F_NOSPLIT)) return "unknown flags";
   switch (w->kind) {
     case SR_WL_DIVLOOP:
       if (w->divloop.fma_count % 8 != 0) return "divloop.fma_count must be a multiple of 8";

@@ -303,8 +303,8 @@ def test_mcml_full_size_invariants(ctx):
     id range equals the oracle."""
     m = I.C3
     nt, it = m.n_threads, m.iters
-    w = mc_workload(m)
-    full = run_mc(ctx, w, nt, it, I.PRIMARY_SEED, sr.SPEC_LOOP, 32, m)
+    w = mc_workload(m, unroll=m.merge_unroll)      # the bench's launch configuration
+    full = run_mc(ctx, w, nt, it, I.PRIMARY_SEED, sr.SPEC_LOOP, m.threshold, m)
     assert full["counters"][0] == nt * it
     for mode, T in ((sr.PDOM, 0), (sr.SPEC_LOOP, 16)):
         o = run_mc(ctx, w, nt, it, I.PRIMARY_SEED, mode, T, m)
@@ -322,4 +322,22 @@ def test_mcml_full_size_invariants(ctx):
     ref = mc_oracle(m, off, 20000, I.PRIMARY_SEED)
     got = run_mc(ctx, mc_workload(m, task_offset=off), 20000, 1, I.PRIMARY_SEED, sr.SPEC_LOOP,
                  32, m)
+    assert_mc_equal(got, ref)
+
+
+@pytest.mark.parametrize("n,iters,off,cap", [
+    (1, 1, 0, 100000),                  # one lane, one photon
+    (33, 2, 0, 100000),                 # one full warp + a 1-lane warp
+    (64, 3, 0, 3),                      # step cap hit by nearly every photon
+    (100, 2, (1 << 40) + 12345, 100000),  # ids above 2^32: the counter's task_hi word
+    (96, 1, 2**64 - 97, 100000),        # top of the 64-bit id space (end = 2^64 - 1)
+])
+@pytest.mark.parametrize("mode,T,U", [(sr.PDOM, 0, 1), (sr.SPEC_LOOP, 32, 4), (sr.SPEC_LOOP, 8, 1)])
+@pytest.mark.parametrize("flags", [0, sr.F_STATIC])
+def test_mcml_edge_cases(ctx, n, iters, off, cap, mode, T, U, flags):
+    import dataclasses
+    m = dataclasses.replace(I.C3, step_cap=cap)
+    ref = mc_oracle(m, off, n * iters, I.PRIMARY_SEED)
+    got = run_mc(ctx, mc_workload(m, task_offset=off, flags=flags, unroll=U), n, iters,
+                 I.PRIMARY_SEED, mode, T, m)
     assert_mc_equal(got, ref)

@@ -78,7 +78,7 @@ def render(ctx, cfg, mode, T, flags=0, block=0):
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 8),
                                     (sr.SPEC_LOOP, 32)])
 @pytest.mark.parametrize("block", [32, 128])
-@pytest.mark.parametrize("flags", [0, sr.F_COARSE])
+@pytest.mark.parametrize("flags", [0, sr.F_COARSE, sr.F_NOSPLIT])
 def test_render_bit_exact_small(ctx, mode, T, block, flags):
     cfg = I.C4_SMALL
     tris, mat, mats, cam, buf, used = scene(cfg)
@@ -94,9 +94,13 @@ def test_render_full_config_invariants_and_sampled_pixels(ctx):
     a, ca = render(ctx, cfg, sr.SPEC_LOOP, 32)
     b, cb = render(ctx, cfg, sr.PDOM, 0)
     c, cc = render(ctx, cfg, sr.SPEC_LOOP, 16, flags=sr.F_COARSE)
+    d, cd = render(ctx, cfg, sr.SPEC_LOOP, 8, flags=sr.F_NOSPLIT)
     assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
     assert np.array_equal(a.view(np.uint32), c.view(np.uint32))
-    assert np.array_equal(ca, cb) and np.array_equal(ca, cc)
+    assert np.array_equal(a.view(np.uint32), d.view(np.uint32))
+    # rays, node visits and triangle tests too: every schedule runs each
+    # lane's traversal in the same order
+    assert np.array_equal(ca, cb) and np.array_equal(ca, cc) and np.array_equal(ca, cd)
     assert ca[0] == cfg.n_pixels * cfg.spp
     tris, mat, mats, cam, buf, used = scene(cfg)
     pix = np.array([0, 1023, 512 * 1024 + 512, 700 * 1024 + 300, 1024 * 1024 - 1, 123457],

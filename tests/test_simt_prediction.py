@@ -15,7 +15,8 @@ sys.path.insert(0, os.path.join(ROOT, "tools"))
 
 CASES = ["divloop_pdom", "divloop_spec(T=16)", "commoncall_pdom", "commoncall_spec",
          "rs_pdom", "rs_spec(T=24)",
-         "mcml_pdom_static", "mcml_spec_static(T=32)", "mcml_spec_static(T=8)"]
+         "mcml_pdom_static", "mcml_spec_static(T=32)", "mcml_spec_static(T=8)",
+         "mcml_spec_static(T=32,U=4)"]
 
 
 @pytest.fixture(scope="module")

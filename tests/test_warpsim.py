@@ -146,9 +146,13 @@ def test_loopmerge_defer_conservation(T, Tb):
     ev, off, ns, ids = _mc_events(K, W, 9)
     r = oracle.ws_loopmerge_defer_raw(ns[ids], ev, off[ids].ravel(), T, Tb)
     nb = int(((ev & oracle.EV_BOUNDARY) != 0).sum())
+    nm = int(((ev & oracle.EV_MATCHED) != 0).sum())    # equal-index boundaries: no part B
+    assert 0 < nm < nb and not ((ev & oracle.EV_MATCHED) & ~((ev & 1) * 0xffff)).any()
     assert r["STEP"][1] == ns.sum()                   # every step runs part A once
-    assert r["B_REL"][1] == nb                        # every boundary sub-step runs once
+    assert r["B_REL"][1] == nb - nm                   # every other boundary sub-step runs once
     assert r["EV0"][1] == nb                          # ... after parking in part A
+    assert r["BI"][1] == nm                           # matched ones finish in part A
+    assert r["A_TAIL"][1] == ns.sum() - (nb - nm)
     assert r["NEV0"][1] == ns.sum() - nb
     assert r["LAUNCH"][1] == W * K
     # the parked set is released in fewer executions than boundary steps

@@ -10,6 +10,9 @@ VARIANTS = {
     "libsr_t768.so": ["SR_MCML_MAXT=768", "SR_MCML_MINB=2"],
     "libsr_t1024.so": ["SR_MCML_MAXT=1024", "SR_MCML_MINB=1"],
     "libsr_t384.so": ["SR_MCML_MAXT=384", "SR_MCML_MINB=3"],
+    "libsr_pts5.so": ["SR_PT_MINB_SPEC=5"],
+    "libsr_pts7.so": ["SR_PT_MINB_SPEC=7"],
+    "libsr_ptp6.so": ["SR_PT_MINB_PDOM=6"],
 }
 if __name__ == "__main__":
     names = sys.argv[1:] or list(VARIANTS)

@@ -17,8 +17,9 @@ M=smsp__thread_inst_executed_per_inst_executed.ratio,smsp__inst_executed.sum,sms
 # every kernel family at its configs[] size (bench launch configuration)
 timeout 1200 ncu --metrics $M --clock-control none -k regex:"divloop|commoncall|mcml|rs_|pt_" --csv --log-file $O/simt_$TAG.csv python tools/one_launch.py > $O/simt_$TAG.log 2>&1
 # the simulator validation launches (static assignment, the oracle replays every warp)
-timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes pdom,spec --threshold 32 > /dev/null 2>&1
-timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic8_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes spec --threshold 8 > /dev/null 2>&1
+timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes pdom,spec --threshold 32 --unroll 1 > /dev/null 2>&1
+timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic8_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes spec --threshold 8 --unroll 1 > /dev/null 2>&1
+timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstaticu4_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes spec --threshold 32 --unroll 4 > /dev/null 2>&1
 # launch list of one short bench run (shares, not absolutes)
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-configs > $O/launches_$TAG.log 2>&1
 # full captures of the dominant kernel (and its PDOM baseline), at 2M photons

@@ -21,6 +21,9 @@ ap.add_argument("--modes", default="pdom,spec")
 ap.add_argument("--threshold", type=int, default=32)
 ap.add_argument("--static", action="store_true")
 ap.add_argument("--iters", type=int, default=0, help="MCML photons per lane (default configs[2]: 64)")
+ap.add_argument("--unroll", type=int, default=I.C3.merge_unroll,
+                help="MCML merge unroll (default: the bench's, configs[2])")
+ap.add_argument("--pt-flags", type=int, default=0, help="extra PATHTRACE flags (F_NOSPLIT = 8)")
 a = ap.parse_args()
 modes = a.modes.split(",")
 ctx = sr.Context.create(0, 1 << 20)
@@ -43,7 +46,7 @@ if "mcml" in a.what:
     iters = a.iters or m.iters
     nt = a.photons // iters
     w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
-                         flags=sr.F_STATIC if a.static else 0)
+                         flags=sr.F_STATIC if a.static else 0, unroll=a.unroll)
     ctx.ensure(sr.sr_workspace_bytes(w, nt))
     for md in modes:
         sr.sr_run(w, nt, iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
@@ -60,7 +63,7 @@ if "pathtrace" in a.what:
     tris, mat, mats, cam = I.cornell_scene(c)
     buf, used = sr.upload_scene(tris, mat, mats, cam)
     w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth,
-                              flags=sr.F_STATIC)
+                              flags=a.pt_flags)
     ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
     for md in modes:
         sr.sr_run(w, c.n_pixels, c.spp, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,

@@ -76,7 +76,7 @@ def commoncall_warps(mode):
 MC_VALIDATION = dict(n_threads=16384, iters=8)   # static launch the oracle can replay
 
 
-def mcml_warps(mode, T, n_threads=MC_VALIDATION["n_threads"], iters=MC_VALIDATION["iters"]):
+def mcml_warps(mode, T, n_threads=MC_VALIDATION["n_threads"], iters=MC_VALIDATION["iters"], U=1):
     m = I.C3
     p = oracle.mc_params(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap)
     ev, off, ns = oracle.mcml_events_batch(p, 0, n_threads * iters, I.PRIMARY_SEED)
@@ -84,7 +84,7 @@ def mcml_warps(mode, T, n_threads=MC_VALIDATION["n_threads"], iters=MC_VALIDATIO
     for w in range(0, n_threads, 32):
         lanes = np.arange(w, min(w + 32, n_threads))
         ids = lanes[:, None] + np.arange(iters)[None, :] * n_threads   # static assignment
-        yield oracle.ws_loopmerge_raw(ns[ids], ev, off[ids].ravel(), mode, T), len(lanes)
+        yield oracle.ws_loopmerge_raw(ns[ids], ev, off[ids].ravel(), mode, T, U=U), len(lanes)
 
 
 def rsbench_warps(mode, T):
@@ -103,6 +103,8 @@ CASES = {
     "mcml_pdom_static": (r"mcml_pdomILb0ELb0", lambda: mcml_warps(oracle.PDOM, 0)),
     "mcml_spec_static(T=32)": (r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 32)),
     "mcml_spec_static(T=8)": (r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 8)),
+    "mcml_spec_static(T=32,U=4)": (r"mcml_specILb0ELb0",
+                                   lambda: mcml_warps(oracle.SPEC_LOOP, 32, U=4)),
     "rs_pdom": (r"rs_pdomILi8ELb0", lambda: rsbench_warps(oracle.PDOM, 0)),
     "rs_spec(T=24)": (r"rs_specILi8ELb0", lambda: rsbench_warps(oracle.SPEC_LOOP, 24)),
 }

@@ -25,6 +25,7 @@ LABELS_ALL = ["divloop_pdom", "divloop_spec(T=16)", "commoncall_pdom", "commonca
               "pt_spec(T=8)"]
 LABELS_MCSTATIC = ["mcml_pdom_static", "mcml_spec_static(T=32)"]
 LABELS_MCSTATIC8 = ["mcml_spec_static(T=8)"]
+LABELS_MCSTATICU4 = ["mcml_spec_static(T=32,U=4)"]
 
 
 def read_ncu_csv(path):
@@ -88,7 +89,8 @@ def main():
     js = {}
     for fname, labels in ((f"simt_{tag}.csv", LABELS_ALL),
                           (f"simt_mcstatic_{tag}.csv", LABELS_MCSTATIC),
-                          (f"simt_mcstatic8_{tag}.csv", LABELS_MCSTATIC8)):
+                          (f"simt_mcstatic8_{tag}.csv", LABELS_MCSTATIC8),
+                          (f"simt_mcstaticu4_{tag}.csv", LABELS_MCSTATICU4)):
         path = os.path.join(OUT, fname)
         if not os.path.exists(path):
             continue
