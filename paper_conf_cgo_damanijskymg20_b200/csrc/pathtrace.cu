@@ -580,7 +580,15 @@ size_t pathtrace_perthread_bytes(uint64_t n) { return 12 * n; }
 static cudaError_t read_header(const void* scene, PtHeader& h) {
   cudaError_t e = cudaMemcpy(&h, scene, sizeof h, cudaMemcpyDeviceToHost);
   if (e != cudaSuccess) return e;
-  if (h.magic != kPtMagic) return cudaErrorInvalidValue;
+  if (h.magic != kPtMagic) {
+    set_launch_note("scene_dev does not hold an sr_scene_build image");
+    return cudaErrorInvalidValue;
+  }
+  if (h.stack_need > kMaxStack) {
+    set_launch_note("scene BVH needs a traversal stack of " + std::to_string(h.stack_need) +
+                    " entries, more than " + std::to_string(kMaxStack));
+    return cudaErrorInvalidValue;
+  }
   return cudaSuccess;
 }
 
@@ -589,7 +597,10 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
   PtHeader h;
   cudaError_t e = read_header(w.pathtrace.scene_dev, h);
   if (e != cudaSuccess) return e;
-  if (h.bytes > w.pathtrace.scene_bytes) return cudaErrorInvalidValue;
+  if (h.bytes > w.pathtrace.scene_bytes) {
+    set_launch_note("pathtrace.scene_bytes is smaller than the scene image");
+    return cudaErrorInvalidValue;
+  }
   PtArgs a = base_args(w.pathtrace.scene_dev);
   a.nodes = reinterpret_cast<const PtNode*>(a.scene + h.off_nodes);
   a.tris = reinterpret_cast<const PtTri*>(a.scene + h.off_tris);
@@ -599,7 +610,6 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
   a.spp = iters;
   a.max_depth = w.pathtrace.max_depth;
   a.unroll = w.pathtrace.merge_unroll ? w.pathtrace.merge_unroll : 8;
-  if (h.stack_need > kMaxStack) return cudaErrorInvalidValue;
   a.stack_cap = h.stack_need > 0 ? h.stack_need : 1u;
   a.T = T;
   a.n = n;
@@ -657,7 +667,6 @@ cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* ray
   a.q_rays = rays;
   a.q_hit = hit;
   a.q_t = t;
-  if (h.stack_need > kMaxStack) return cudaErrorInvalidValue;
   a.stack_cap = h.stack_need > 0 ? h.stack_need : 1u;
   const unsigned grid = (unsigned)((n + 127) / 128);
   record_launch(grid, 128, 0);

@@ -35,10 +35,13 @@ int fail(int code, const std::string& msg) {
   g_err = msg;
   return code;
 }
+thread_local std::string g_note;  // launcher's explanation of its own error return
 int fail_cuda(cudaError_t e, const char* where) {
   cudaGetLastError();  // clear sticky-free errors
-  return fail(SR_E_CUDA, std::string(where) + ": " + cudaGetErrorName(e) + ": " +
-                             cudaGetErrorString(e));
+  std::string msg = std::string(where) + ": " + cudaGetErrorName(e) + ": " + cudaGetErrorString(e);
+  if (!g_note.empty()) msg += " (" + g_note + ")";
+  g_note.clear();
+  return fail(SR_E_CUDA, msg);
 }
 size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
 
@@ -132,6 +135,8 @@ Layout layout_of(const sr_workload& w, uint64_t n) {
   L.total = off;
   return L;
 }
+
+void set_launch_note(const std::string& why) { g_note = why; }
 
 }  // namespace sr
 

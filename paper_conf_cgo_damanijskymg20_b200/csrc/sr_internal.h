@@ -32,6 +32,10 @@ struct LaunchCtx {
 // Set the calling thread's sr_last_error() text; returns `code`.
 int set_error(int code, const std::string& msg);
 
+// A launcher returning an error of its own (not the driver's) explains it
+// here; the text is appended to sr_last_error().
+void set_launch_note(const std::string& why);
+
 // The launch configuration of the most recent kernel (sr_last_launch).
 void record_launch(uint32_t grid, uint32_t block, uint32_t smem_bytes);
 
