@@ -131,3 +131,43 @@ def test_event_stream_matches_step_counts():
         assert (ev[0] & oracle.EV_SLEFT) == 0
         # only the last step can exit
         assert np.all((ev[:-1] & oracle.EV_EXIT) == 0)
+
+
+def test_equal_layers_equal_one_slab():
+    """A slab cut into three layers with identical optics scatters light exactly
+    like the uncut slab (an internal boundary between equal indices is not
+    physical: Fresnel r = 0, the step continues with its leftover length, MCML
+    ref. [2] of the paper).  Pins the layer-crossing code -- leftover path
+    length, layer index, the matched-boundary branch -- statistically: Rd, Tt
+    and the absorbed weight per depth band agree within 5 sigma (sigma the
+    [0,1]-bounded-mean bound sqrt(p(1-p)/N), doubled for the difference)."""
+    n_, mua, mus, g = 1.4, 2.0, 98.0, 0.8
+    one = I.MCML(layers=((n_, mua, mus, g, 0.06),), nz=60, dz=0.001)
+    three = I.MCML(layers=((n_, mua, mus, g, 0.02),) * 3, nz=60, dz=0.001)
+    N = 200000
+    a = oracle.mcml(P(one), 0, N, I.PRIMARY_SEED)
+    b = oracle.mcml(P(three), 0, N, I.PRIMARY_SEED)
+    ev = np.concatenate([oracle.mcml_events(P(three), k, I.PRIMARY_SEED) for k in range(200)])
+    assert ((ev & oracle.EV_MATCHED) != 0).sum() > 0     # the crossings happen
+    bands = lambda o: o["A"].sum(axis=1).reshape(6, 10).sum(axis=1)
+    for qa, qb in [(a["Rd"].sum(), b["Rd"].sum()), (a["Tt"].sum(), b["Tt"].sum()),
+                   *zip(bands(a), bands(b))]:
+        pa, pb = qa / FX / N, qb / FX / N
+        sig = math.sqrt(max(pa, 1e-6) * (1 - pa) / N)
+        assert abs(pa - pb) < 2 * 5 * sig, (pa, pb)
+
+
+def test_matched_boundary_events():
+    """MATCHED marks exactly the boundary steps between layers of equal index:
+    never an exit, always a reflect or a transmit, and only inside the slab."""
+    p = P(I.C3)
+    for k in range(50):
+        ev = oracle.mcml_events(p, k, I.PRIMARY_SEED).astype(np.int64)
+        m = (ev & oracle.EV_MATCHED) != 0
+        assert np.all((ev[m] & oracle.EV_BOUNDARY) != 0)
+        assert np.all((ev[m] & (oracle.EV_EXIT | oracle.EV_EXTERNAL)) == 0)
+        assert np.all(np.isin(ev[m] & (oracle.EV_REFLECT | oracle.EV_TRANSMIT), [4, 16]))
+    # configs[2] has equal indices throughout: every internal crossing is matched
+    ev = np.concatenate([oracle.mcml_events(p, k, I.PRIMARY_SEED) for k in range(300)]).astype(np.int64)
+    internal = ((ev & oracle.EV_BOUNDARY) != 0) & ((ev & oracle.EV_EXTERNAL) == 0)
+    assert np.array_equal(internal, (ev & oracle.EV_MATCHED) != 0)
