@@ -227,13 +227,27 @@ SR_API int sr_pt_closest(const void* scene_dev, const float* rays_dev, int64_t* 
  *   mat        host, n_tris x uint32 material ids (< n_mats)
  *   mats       host, n_mats x 8 floats {kind, r, g, b, er, eg, eb, ior}
  *              kind: 0 diffuse, 1 mirror, 2 dielectric, 3 emissive-only
- *   cam        host, 12 floats {eye xyz, look-at xyz, up xyz, tan(fov/2), 0, 0}
+ *   cam        host, 14 floats {eye xyz, forward xyz, right xyz, up xyz (an
+ *              orthonormal basis), tan(fov/2), aspect = width/height}
  *   dst_dev    device buffer of dst_bytes; *needed receives the size.  If
- *              dst_dev is NULL only *needed is computed.
- * The BVH is deterministic for a given input. */
+ *              dst_dev is NULL only *needed is computed (an upper bound; after
+ *              a build, the exact image size).
+ * The image (pt_scene.h layout: header, two-wide BVH nodes, triangles in BVH
+ * order, materials) is deterministic for a given input.  The header records
+ * the deepest traversal stack a ray can need; the PATHTRACE kernels reject a
+ * scene needing more than 256 entries.  Errors: SR_E_INVALID (NULL inputs,
+ * n_tris = 0 or >= 2^31, material id >= n_mats, material kind not 0..3,
+ * non-finite vertices),
+ * SR_E_NOMEM (dst_bytes < *needed), SR_E_CUDA (the copy failed). */
 SR_API int sr_scene_build(const float* tris, const uint32_t* mat, uint32_t n_tris, const float* mats,
                    uint32_t n_mats, const float* cam, void* dst_dev, size_t dst_bytes,
                    size_t* needed);
+
+/* The same build into HOST memory (dst_host): no device, no context needed --
+ * for inspecting / validating the BVH on the CPU. */
+SR_API int sr_scene_build_host(const float* tris, const uint32_t* mat, uint32_t n_tris,
+                               const float* mats, uint32_t n_mats, const float* cam,
+                               void* dst_host, size_t dst_bytes, size_t* needed);
 
 #ifdef __cplusplus
 }

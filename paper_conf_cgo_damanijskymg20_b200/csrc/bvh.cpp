@@ -170,8 +170,12 @@ size_t image_bound(uint32_t n_tris, uint32_t n_mats) {
 std::string check_scene_inputs(const float* tris, const uint32_t* mat, uint32_t n_tris,
                                const float* mats, uint32_t n_mats, const float* cam) {
   if (n_tris == 0) return "n_tris must be >= 1";
+  if (n_tris >= (1u << 31)) return "n_tris must be < 2^31 (BVH references are int32)";
   if (!tris || !mat || !mats || !cam) return "NULL input array";
   if (n_mats == 0) return "n_mats must be >= 1";
+  for (size_t i = 0; i < 9 * (size_t)n_tris; ++i)
+    if (!std::isfinite(tris[i])) return "non-finite vertex coordinate at triangle " +
+                                        std::to_string(i / 9);
   for (uint32_t i = 0; i < n_tris; ++i)
     if (mat[i] >= n_mats) return "material id out of range at triangle " + std::to_string(i);
   for (uint32_t m = 0; m < n_mats; ++m) {
@@ -186,16 +190,18 @@ std::string check_scene_inputs(const float* tris, const uint32_t* mat, uint32_t 
 
 using namespace sr;
 
-extern "C" int sr_scene_build(const float* tris, const uint32_t* mat, uint32_t n_tris,
-                              const float* mats, uint32_t n_mats, const float* cam, void* dst_dev,
-                              size_t dst_bytes, size_t* needed) {
+// Builds the scene image; copies it to dst with cudaMemcpy (device) or memcpy
+// (host).  Shared by sr_scene_build and sr_scene_build_host.
+static int build_scene(const char* fn, bool to_device, const float* tris, const uint32_t* mat,
+                       uint32_t n_tris, const float* mats, uint32_t n_mats, const float* cam,
+                       void* dst, size_t dst_bytes, size_t* needed) {
   if (needed) *needed = 0;
   const std::string why = check_scene_inputs(tris, mat, n_tris, mats, n_mats, cam);
-  if (!why.empty()) return set_error(SR_E_INVALID, "sr_scene_build: " + why);
+  if (!why.empty()) return set_error(SR_E_INVALID, std::string(fn) + ": " + why);
   const size_t bound = image_bound(n_tris, n_mats);
   if (needed) *needed = bound;
-  if (!dst_dev) return SR_OK;
-  if (dst_bytes < bound) return set_error(SR_E_NOMEM, "sr_scene_build: dst_bytes < needed");
+  if (!dst) return SR_OK;
+  if (dst_bytes < bound) return set_error(SR_E_NOMEM, std::string(fn) + ": dst_bytes < needed");
 
   Builder B;
   B.tris = tris;
@@ -304,9 +310,27 @@ extern "C" int sr_scene_build(const float* tris, const uint32_t* mat, uint32_t n
     o.pad = 0;
   }
   std::memcpy(img.data() + h.off_mats, mats, (size_t)n_mats * sizeof(PtMat));
-  const cudaError_t e = cudaMemcpy(dst_dev, img.data(), h.bytes, cudaMemcpyHostToDevice);
-  if (e != cudaSuccess)
-    return set_error(SR_E_CUDA, std::string("sr_scene_build: cudaMemcpy: ") + cudaGetErrorString(e));
+  if (to_device) {
+    const cudaError_t e = cudaMemcpy(dst, img.data(), h.bytes, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess)
+      return set_error(SR_E_CUDA, std::string(fn) + ": cudaMemcpy: " + cudaGetErrorString(e));
+  } else {
+    std::memcpy(dst, img.data(), h.bytes);
+  }
   if (needed) *needed = h.bytes;
   return SR_OK;
+}
+
+extern "C" int sr_scene_build(const float* tris, const uint32_t* mat, uint32_t n_tris,
+                              const float* mats, uint32_t n_mats, const float* cam, void* dst_dev,
+                              size_t dst_bytes, size_t* needed) {
+  return build_scene("sr_scene_build", true, tris, mat, n_tris, mats, n_mats, cam, dst_dev,
+                     dst_bytes, needed);
+}
+
+extern "C" int sr_scene_build_host(const float* tris, const uint32_t* mat, uint32_t n_tris,
+                                   const float* mats, uint32_t n_mats, const float* cam,
+                                   void* dst_host, size_t dst_bytes, size_t* needed) {
+  return build_scene("sr_scene_build_host", false, tris, mat, n_tris, mats, n_mats, cam,
+                     dst_host, dst_bytes, needed);
 }

@@ -27,7 +27,7 @@ MC_COUNTERS = ["photons", "steps", "rd_exits", "tt_exits", "rr_kills", "rr_survi
                "zero_w"]
 EXPORTS = ["sr_init", "sr_workspace_bytes", "sr_workspace_region", "sr_run", "sr_tally",
            "sr_finalize", "sr_last_error", "sr_build_info", "sr_last_launch", "sr_math_eval",
-           "sr_pt_closest", "sr_scene_build"]
+           "sr_pt_closest", "sr_scene_build", "sr_scene_build_host"]
 PT_COUNTERS = ["paths", "rays", "node_visits", "tri_tests"]
 FN_LOGF, FN_SIN2PI, FN_COS2PI, FN_EXPENSIVE_1000, FN_EXPENSIVE_2000 = 0, 1, 2, 3, 4
 
@@ -107,8 +107,9 @@ def load(path: str | None = None):
     L.sr_pt_closest.restype = C.c_int
     fp, up = C.POINTER(C.c_float), C.POINTER(C.c_uint32)
     L.sr_scene_build.argtypes = [fp, up, u32, fp, u32, fp, vp, sz, C.POINTER(sz)]
+    L.sr_scene_build_host.argtypes = [fp, up, u32, fp, u32, fp, vp, sz, C.POINTER(sz)]
     for name in ("sr_init", "sr_workspace_region", "sr_run", "sr_tally", "sr_finalize",
-                 "sr_last_launch", "sr_scene_build"):
+                 "sr_last_launch", "sr_scene_build", "sr_scene_build_host"):
         getattr(L, name).restype = C.c_int
     _lib = L
     return L
@@ -171,17 +172,29 @@ def sr_last_launch() -> dict:
     return {"grid": out[0], "block": out[1], "smem": out[2], "kernels": out[3]}
 
 
-def sr_scene_build(tris, mat, mats, cam, dst_ptr: int | None, dst_bytes: int) -> int:
-    """numpy float32 tris[n,9], uint32 mat[n], float32 mats[m,8], float32 cam[12]."""
+def sr_scene_build(tris, mat, mats, cam, dst_ptr: int | None, dst_bytes: int,
+                   host: bool = False) -> int:
+    """numpy float32 tris[n,9], uint32 mat[n], float32 mats[m,8], float32 cam[14];
+    dst_ptr: device address (sr_scene_build) or, with host=True, a host address
+    (sr_scene_build_host).  Returns the bytes needed / written."""
     import numpy as np
     tris = np.ascontiguousarray(tris, np.float32); mat = np.ascontiguousarray(mat, np.uint32)
     mats = np.ascontiguousarray(mats, np.float32); cam = np.ascontiguousarray(cam, np.float32)
     fp, up = C.POINTER(C.c_float), C.POINTER(C.c_uint32)
     needed = C.c_size_t()
-    _check(load().sr_scene_build(tris.ctypes.data_as(fp), mat.ctypes.data_as(up), len(mat),
-                                 mats.ctypes.data_as(fp), len(mats), cam.ctypes.data_as(fp),
-                                 dst_ptr, dst_bytes, C.byref(needed)))
+    fn = load().sr_scene_build_host if host else load().sr_scene_build
+    _check(fn(tris.ctypes.data_as(fp), mat.ctypes.data_as(up), len(mat), mats.ctypes.data_as(fp),
+              len(mats), cam.ctypes.data_as(fp), dst_ptr, dst_bytes, C.byref(needed)))
     return needed.value
+
+
+def scene_image_host(tris, mat, mats, cam):
+    """The scene image built on the host (numpy uint8), for inspection."""
+    import numpy as np
+    need = sr_scene_build(tris, mat, mats, cam, None, 0, host=True)
+    img = np.zeros(need, np.uint8)
+    used = sr_scene_build(tris, mat, mats, cam, img.ctypes.data, need, host=True)
+    return img[:used]
 
 
 # ------------------------------------------------------------------ workload builders
