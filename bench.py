@@ -430,6 +430,18 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
     res["speedup_vs_pdom"] = res[f"spec_t{c.threshold}"]["value"] / res["pdom"]["value"]
     out["rsbench"] = res
 
+    # ... with an expensive task fetch (2048-FMA prolog, Fig. 9's XSBench case):
+    # refilling idle lanes costs more, the best threshold drops (T = 32 shown too)
+    c = I.NEXT1_FETCH
+    w = sr.rsbench_workload(c.fma_count, prolog_fma=c.prolog_fma)
+    res = {"prolog_fma": c.prolog_fma}
+    for name, mode, thr in (("pdom", sr.PDOM, 0), (f"spec_t{c.threshold}", sr.SPEC_LOOP,
+                                                   c.threshold), ("spec_t32", sr.SPEC_LOOP, 32)):
+        t = graph_time(w, c.n_threads, c.iters, mode, thr, reps=5)
+        res[name] = {"value": c.n_threads * c.iters / (t * 1e-3), "unit": "lookups/s", "ms": t}
+    res["speedup_vs_pdom"] = res[f"spec_t{c.threshold}"]["value"] / res["pdom"]["value"]
+    out["rsbench_fetch"] = res
+
     # configs[3]: path tracer, 1024^2 x 16 spp over the 1,044,494-triangle BVH scene
     c = I.C4
     tris, mat, mats, cam = I.cornell_scene(c)

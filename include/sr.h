@@ -119,7 +119,9 @@ typedef struct {
 
 typedef struct {
   uint32_t fma_count;  /* FMAs of the per-nuclide body; multiple of 8 (64)       */
-  uint32_t reserved;   /* must be 0                                              */
+  uint32_t prolog_fma; /* FMAs of the lookup prolog (an expensive task fetch,
+                          E = Expensive(E, prolog_fma)); multiple of 8, <= 65536;
+                          0 = none (configs: 0; the Fig. 9 XSBench-like sweep: 2048) */
 } sr_rsbench_params;   /* materials / nuclide counts: DESIGN.md reading R8       */
 
 typedef struct {

@@ -168,15 +168,15 @@ def commoncall(t0, n, iters, seed, split_u32=1 << 31, fma_count=2000):
 RS_MATS, RS_NUCLIDES = 12, 355
 
 
-def rsbench(t0, n, iters, seed, fma_count=64, trips=False):
+def rsbench(t0, n, iters, seed, fma_count=64, trips=False, prolog_fma=0):
     L = lib()
     u32p, f32p = C.POINTER(C.c_uint32), C.POINTER(C.c_float)
-    L.or_rsbench.argtypes = [C.c_uint32, C.c_uint64, C.c_uint64, C.c_uint32, C.c_uint64, f32p,
-                             u32p, u32p]
+    L.or_rsbench.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64, C.c_uint64, C.c_uint32,
+                             C.c_uint64, f32p, u32p, u32p]
     acc = np.zeros(n, np.float32); nuc = np.zeros(n, np.uint32)
     tr = np.zeros(n * iters, np.uint32) if trips else None
-    L.or_rsbench(fma_count, t0, n, iters, seed, _p(acc, C.c_float), _p(nuc, C.c_uint32),
-                 _p(tr, C.c_uint32) if trips else None)
+    L.or_rsbench(fma_count, prolog_fma, t0, n, iters, seed, _p(acc, C.c_float),
+                 _p(nuc, C.c_uint32), _p(tr, C.c_uint32) if trips else None)
     return (acc, nuc, tr.reshape(n, iters)) if trips else (acc, nuc)
 
 

@@ -130,9 +130,10 @@ uint32_t or_rs_threshold(uint32_t m);  /* cumulative 2^-32 selection bound   */
 uint32_t or_rs_pick(uint32_t u);       /* material of a Philox word          */
 float or_rs_body(float E, uint32_t nuc, uint32_t fma_count);
 /* per thread: acc = sum over lookups of sum over nuclides of body(); nuc =
- * nuclides visited; trips[j*iters+k] (may be NULL) = inner trip count */
-void or_rsbench(uint32_t fma_count, uint64_t t0, uint64_t n, uint32_t iters, uint64_t seed,
-                float* acc, uint32_t* nuc, uint32_t* trips);
+ * nuclides visited; trips[j*iters+k] (may be NULL) = inner trip count;
+ * prolog_fma > 0: the prolog computes E = or_expensive(E, prolog_fma) */
+void or_rsbench(uint32_t fma_count, uint32_t prolog_fma, uint64_t t0, uint64_t n,
+                uint32_t iters, uint64_t seed, float* acc, uint32_t* nuc, uint32_t* trips);
 
 /* ---- warpsim.c : lane-mask warp simulator (oracle part 2). */
 enum { WS_PDOM = 0, WS_SPEC_LOOP = 1, WS_SPEC_CALL = 2 };

@@ -18,6 +18,11 @@
  * as 2^-32 integer thresholds), nuclide ids n = (37 m + 13 j) mod 355, the
  * per-nuclide body = 8 FMA chains x (fma_count/8) rounds started from
  * (E + n/512), and the epilog acc = acc + xs.
+ *
+ * prolog_fma > 0: the lookup's prolog also does prolog_fma FMAs of work on the
+ * energy, E = Expensive(U01(u1), prolog_fma) (reading R8'): an expensive task
+ * fetch, XSBench's energy-grid search, the case where Fig. 9 finds the best
+ * threshold far below full reconvergence.
  */
 #include <math.h>
 #include "oracle.h"
@@ -49,8 +54,9 @@ float or_rs_body(float E, uint32_t nuc, uint32_t fma_count) {
   return or_expensive(start, fma_count);
 }
 
-void or_rsbench(uint32_t fma_count, uint64_t t0, uint64_t n, uint32_t iters, uint64_t seed,
-                float* acc_out, uint32_t* nuc_out, uint32_t* trips /* may be NULL */) {
+void or_rsbench(uint32_t fma_count, uint32_t prolog_fma, uint64_t t0, uint64_t n,
+                uint32_t iters, uint64_t seed, float* acc_out, uint32_t* nuc_out,
+                uint32_t* trips /* may be NULL */) {
   uint32_t key[2] = {(uint32_t)seed, (uint32_t)(seed >> 32)};
   for (uint64_t j = 0; j < n; ++j) {
     uint64_t t = t0 + j;
@@ -62,6 +68,7 @@ void or_rsbench(uint32_t fma_count, uint64_t t0, uint64_t n, uint32_t iters, uin
       or_philox4x32_10(ctr, key, u);                 /* Prolog */
       uint32_t m = or_rs_pick(u[0]);
       float E = or_u01(u[1]);
+      if (prolog_fma) E = or_expensive(E, prolog_fma);
       float xs = 0.0f;
       uint32_t N = kNucs[m];
       for (uint32_t i = 0; i < N; ++i) {             /* inner loop, L1 */

@@ -33,6 +33,7 @@ struct RsArgs {
   RoundKeys keys;
   uint32_t thr[kMats];   // cumulative selection thresholds (host-computed)
   uint32_t iters, rounds, T;
+  uint32_t prolog_rounds;  // expensive prolog (task fetch): 0 = none
   uint2* out;            // {acc bits, nuclides}
   unsigned long long* counters;
   uint32_t* sched;
@@ -44,6 +45,16 @@ __device__ __forceinline__ uint32_t pick(const RsArgs& a, uint32_t u) {
   for (int i = kMats - 2; i >= 0; --i)
     if (u < a.thr[i]) m = (uint32_t)i;
   return m;
+}
+
+// Prolog energy: U01(u1), or Expensive() of it for an expensive task fetch.
+// PROLOG > 0: compile-time rounds; 0: none; < 0: a.prolog_rounds at run time.
+template <int PROLOG>
+__device__ __forceinline__ float energy(const RsArgs& a, uint32_t u1) {
+  const float E = u01(u1);
+  if constexpr (PROLOG > 0) return expensive<PROLOG>(E, 0u);
+  else if constexpr (PROLOG < 0) return a.prolog_rounds ? expensive<0>(E, a.prolog_rounds) : E;
+  else return E;
 }
 
 template <int ROUNDS>
@@ -68,7 +79,7 @@ __device__ __forceinline__ void finish(const RsArgs& a, uint64_t g, bool valid, 
   }
 }
 
-template <int ROUNDS, bool SCHED>
+template <int ROUNDS, int PROLOG, bool SCHED>
 __global__ void __launch_bounds__(256) rs_pdom(const RsArgs a) {
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
   const bool valid = g < a.n;
@@ -81,7 +92,7 @@ __global__ void __launch_bounds__(256) rs_pdom(const RsArgs a) {
     if (valid) {
       const uint4 u = draw(k, kTagRs, t, a.keys);  // @sr-region LAUNCH
       m = pick(a, u.x);
-      E = u01(u.y);
+      E = energy<PROLOG>(a, u.y);
       N = c_nucs[m];
     }
     float xs = 0.0f;
@@ -101,7 +112,7 @@ __global__ void __launch_bounds__(256) rs_pdom(const RsArgs a) {
   finish(a, g, valid, acc, nucs, a.iters, r, rl, a.iters, a.iters * (uint32_t)__popc(__ballot_sync(kFull, valid)));
 }  // @sr-region END
 
-template <int ROUNDS, bool SCHED>
+template <int ROUNDS, int PROLOG, bool SCHED>
 __global__ void __launch_bounds__(256) rs_spec(const RsArgs a) {
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
   const bool valid = g < a.n;
@@ -133,7 +144,7 @@ __global__ void __launch_bounds__(256) rs_spec(const RsArgs a) {
       if ((R >> lane_id()) & 1u) {
         const uint4 u = draw(k, kTagRs, t, a.keys);  // @sr-region LAUNCH
         m = pick(a, u.x);
-        E = u01(u.y);
+        E = energy<PROLOG>(a, u.y);
         N = c_nucs[m];
         i = 0;
         xs = 0.0f;
@@ -153,11 +164,14 @@ cudaError_t launch_t(const LaunchCtx& c, const RsArgs& a, int mode) {
   if (grid > 0x7fffffffull) return cudaErrorInvalidConfiguration;
   record_launch((uint32_t)grid, block, 0);
   const bool spec = mode == SR_SPEC_LOOP;
-#define SR_RS(R)                                                                    \
-  (spec ? rs_spec<R, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a)            \
-        : rs_pdom<R, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a))
-  if (a.rounds == 8) SR_RS(8);
-  else SR_RS(0);
+#define SR_RS(R, PR)                                                                \
+  (spec ? rs_spec<R, PR, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a)        \
+        : rs_pdom<R, PR, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a))
+  // compile-time shapes of the measured configurations (straight-line code,
+  // static SASS costs for the simulator); anything else runs the generic one
+  if (a.rounds == 8 && a.prolog_rounds == 0) SR_RS(8, 0);
+  else if (a.rounds == 8 && a.prolog_rounds == 256) SR_RS(8, 256);
+  else SR_RS(0, -1);
 #undef SR_RS
   return cudaGetLastError();
 }
@@ -180,6 +194,7 @@ cudaError_t launch_rsbench(const LaunchCtx& c, const sr_workload& w, uint64_t n,
   a.keys = round_keys(seed);
   a.iters = iters;
   a.rounds = w.rsbench.fma_count / 8u;
+  a.prolog_rounds = w.rsbench.prolog_fma / 8u;
   a.T = T;
   a.out = reinterpret_cast<uint2*>(c.ws + c.lay.off[SR_T_PERTHREAD]);
   a.counters = reinterpret_cast<unsigned long long*>(c.ws + c.lay.off[SR_T_COUNTERS]);

@@ -67,7 +67,8 @@ std::string check_workload(const sr_workload* w, uint64_t n_threads) {
       return check_pathtrace(w->pathtrace, n_threads);
     case SR_WL_RSBENCH:
       if (w->rsbench.fma_count % 8 != 0) return "rsbench.fma_count must be a multiple of 8";
-      if (w->rsbench.reserved != 0) return "rsbench.reserved must be 0";
+      if (w->rsbench.prolog_fma % 8 != 0 || w->rsbench.prolog_fma > 65536)
+        return "rsbench.prolog_fma must be a multiple of 8 in [0, 65536]";
       if (n_threads > (1ull << 40)) return "n_threads too large";
       return "";
     default:

@@ -41,9 +41,14 @@ class RSBench:
     iters: int = 32             # lookups per thread (thread coarsening)
     fma_count: int = 64         # FMAs of the per-nuclide body
     threshold: int = 24         # best of the sweep (profiles/threshold_sweep_*.md)
+    prolog_fma: int = 0         # FMAs of the lookup prolog (expensive task fetch)
 
 
 NEXT1 = RSBench()
+# Fig. 9's XSBench case: an expensive task fetch (2048 FMAs per
+# lookup prolog, ~0.6x the mean inner-loop work of a lookup) -- refilling idle
+# lanes often no longer pays, the best threshold drops
+NEXT1_FETCH = RSBench(prolog_fma=2048, threshold=12)   # best of the sweep
 
 
 # (n, mua [1/cm], mus [1/cm], g, d [cm]) -- a synthetic 3-layer tissue slab

@@ -64,7 +64,7 @@ class PathtraceParams(C.Structure):
 
 
 class RsbenchParams(C.Structure):
-    _fields_ = [("fma_count", C.c_uint32), ("reserved", C.c_uint32)]
+    _fields_ = [("fma_count", C.c_uint32), ("prolog_fma", C.c_uint32)]
 
 
 class Workload(C.Structure):
@@ -204,9 +204,9 @@ def divloop_workload(p_u32=1 << 29, fma_count=1000, task_offset=0, flags=0, bloc
     return w
 
 
-def rsbench_workload(fma_count=64, task_offset=0, flags=0, block=0) -> Workload:
+def rsbench_workload(fma_count=64, task_offset=0, flags=0, block=0, prolog_fma=0) -> Workload:
     w = Workload(kind=WL_RSBENCH, flags=flags, task_offset=task_offset, block_threads=block)
-    w.rsbench = RsbenchParams(fma_count, 0)
+    w.rsbench = RsbenchParams(fma_count, prolog_fma)
     return w
 
 

@@ -72,3 +72,29 @@ def test_rsbench_full_config_sampled(ctx):
     for t in rng.choice(c.n_threads, 64, replace=False):
         acc_o, nuc_o = oracle.rsbench(int(t), 1, c.iters, I.PRIMARY_SEED, c.fma_count)
         assert a_spec[t].view(np.uint32) == acc_o[0].view(np.uint32) and n_spec[t] == nuc_o[0]
+
+
+@pytest.mark.parametrize("prolog", [256, 2048, 8])   # generic, compile-time, smallest
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 4), (sr.SPEC_LOOP, 16),
+                                    (sr.SPEC_LOOP, 32)])
+def test_rsbench_expensive_prolog_bit_exact(ctx, prolog, mode, T):
+    """The expensive-task-fetch variant (Fig. 9's XSBench case): every mode and
+    threshold equals the oracle bit for bit, also in the schedule counters'
+    kernels (the prolog does not change the trip counts)."""
+    n, iters = 333, 5
+    acc_o, nuc_o = oracle.rsbench(7, n, iters, I.PRIMARY_SEED, prolog_fma=prolog)
+    w = sr.rsbench_workload(block=96, task_offset=7, prolog_fma=prolog)
+    acc, nuc, cnt = run(ctx, w, n, iters, I.PRIMARY_SEED, mode, T)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(nuc, nuc_o)
+
+
+def test_rsbench_expensive_prolog_full_config_sampled(ctx):
+    c = I.NEXT1_FETCH
+    w = sr.rsbench_workload(c.fma_count, prolog_fma=c.prolog_fma)
+    a, nn, _ = run(ctx, w, c.n_threads, c.iters, I.PRIMARY_SEED, sr.SPEC_LOOP, c.threshold)
+    rng = np.random.default_rng(2)
+    for t in rng.choice(c.n_threads, 16, replace=False):
+        acc_o, nuc_o = oracle.rsbench(int(t), 1, c.iters, I.PRIMARY_SEED, c.fma_count,
+                                      prolog_fma=c.prolog_fma)
+        assert a[t].view(np.uint32) == acc_o[0].view(np.uint32) and nn[t] == nuc_o[0]

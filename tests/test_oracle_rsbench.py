@@ -59,3 +59,21 @@ def test_thread_sums_within_closed_form_range():
     hi = expensive_closed_form(1.0 + 354 * 2.0**-9, 64) + expensive_tol(64)
     per = acc / nuc
     assert per.min() >= lo * (1 - 1e-5) and per.max() <= hi * (1 + 1e-5)
+
+
+def test_expensive_prolog_changes_energies_not_trips():
+    """prolog_fma (reading R8'): the lookup prolog computes E = Expensive(U01,
+    prolog_fma); trip counts are untouched and every per-nuclide value lies in
+    the closed-form range of a body started from the prolog's range."""
+    n, it = 300, 4
+    _, nuc0, tr0 = oracle.rsbench(0, n, it, 3, fma_count=64, trips=True)
+    acc, nuc, tr = oracle.rsbench(0, n, it, 3, fma_count=64, trips=True, prolog_fma=2048)
+    assert np.array_equal(nuc, nuc0) and np.array_equal(tr, tr0)
+    e_lo = expensive_closed_form(0.0, 2048) - expensive_tol(2048)
+    e_hi = expensive_closed_form(1.0, 2048) + expensive_tol(2048)
+    lo = expensive_closed_form(e_lo, 64) - expensive_tol(64)
+    hi = expensive_closed_form(e_hi + 354 * 2.0**-9, 64) + expensive_tol(64)
+    per = acc / nuc
+    assert per.min() >= lo * (1 - 1e-5) and per.max() <= hi * (1 + 1e-5)
+    acc_plain, _ = oracle.rsbench(0, n, it, 3, fma_count=64)
+    assert not np.array_equal(acc, acc_plain)

@@ -16,7 +16,7 @@ simulated in full at their configs[] size.
 
 TEST/EVALUATION INFRASTRUCTURE: uses oracle/ (event streams + simulator).
 
-usage: python tools/select_threshold.py [--what divloop,rsbench,mcml]
+usage: python tools/select_threshold.py [--what divloop,rsbench,rsfetch,mcml]
            [--thresholds 1,2,4,8,16,24,32] [--mc-warps 512] [--mc-iters 64]
            [--unroll 4] [--measured sweep.json ...] [--write out.json]
 """
@@ -58,7 +58,7 @@ def mc_warps(sample, iters, mode, T, U):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--what", default="divloop,rsbench,mcml")
+    ap.add_argument("--what", default="divloop,rsbench,rsfetch,mcml")
     ap.add_argument("--thresholds", default="1,2,4,8,16,24,32")
     ap.add_argument("--mc-warps", type=int, default=512)
     ap.add_argument("--mc-iters", type=int, default=I.C3.iters)
@@ -74,7 +74,11 @@ def main():
         fams["divloop"] = (r"divloop_pdomILi125ELb0", r"divloop_specILi125ELb0",
                            lambda mode, T: sp.divloop_warps(mode, T), I.C1.n_threads * I.C1.iters)
     if "rsbench" in a.what:
-        fams["rsbench"] = (r"rs_pdomILi8ELb0", r"rs_specILi8ELb0",
+        fams["rsbench"] = (r"rs_pdomILi8ELi0ELb0", r"rs_specILi8ELi0ELb0",
+                           lambda mode, T: sp.rsbench_warps(mode, T),
+                           I.NEXT1.n_threads * I.NEXT1.iters)
+    if "rsfetch" in a.what:   # the expensive-prolog variant (trip counts are the same)
+        fams["rsfetch"] = (r"rs_pdomILi8ELi256ELb0", r"rs_specILi8ELi256ELb0",
                            lambda mode, T: sp.rsbench_warps(mode, T),
                            I.NEXT1.n_threads * I.NEXT1.iters)
     if "mcml" in a.what:

@@ -105,8 +105,8 @@ CASES = {
     "mcml_spec_static(T=8)": (r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 8)),
     "mcml_spec_static(T=32,U=4)": (r"mcml_specILb0ELb0",
                                    lambda: mcml_warps(oracle.SPEC_LOOP, 32, U=4)),
-    "rs_pdom": (r"rs_pdomILi8ELb0", lambda: rsbench_warps(oracle.PDOM, 0)),
-    "rs_spec(T=24)": (r"rs_specILi8ELb0", lambda: rsbench_warps(oracle.SPEC_LOOP, 24)),
+    "rs_pdom": (r"rs_pdomILi8ELi0ELb0", lambda: rsbench_warps(oracle.PDOM, 0)),
+    "rs_spec(T=24)": (r"rs_specILi8ELi0ELb0", lambda: rsbench_warps(oracle.SPEC_LOOP, 24)),
 }
 
 

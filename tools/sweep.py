@@ -28,6 +28,7 @@ ap.add_argument("--unroll", type=int, default=0, help="PT node-merge partial unr
 ap.add_argument("--defer", type=int, default=0, help="MCML boundary defer threshold T_b")
 ap.add_argument("--static", action="store_true", help="MCML static photon assignment (F_STATIC)")
 ap.add_argument("--iters", type=int, default=0, help="MCML photons per lane (default configs[2])")
+ap.add_argument("--prolog", type=int, default=0, help="RSBench prolog FMAs (expensive task fetch)")
 a = ap.parse_args()
 Ts = [int(x) for x in a.thresholds.split(",")]
 blocks = [int(x) for x in a.blocks.split(",")]
@@ -105,7 +106,7 @@ if "rsbench" in a.what:
     c = I.NEXT1
     res = []
     for b in blocks:
-        w = sr.rsbench_workload(c.fma_count, block=b)
+        w = sr.rsbench_workload(c.fma_count, block=b, prolog_fma=a.prolog)
         ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
             t = timed(lambda: sr.sr_run(w, c.n_threads, c.iters, seed, mode, T), a.reps)
@@ -114,7 +115,7 @@ if "rsbench" in a.what:
             r.update(eff(w, c.n_threads, c.iters, mode, T))
             res.append(r)
             print(json.dumps(r), file=sys.stderr, flush=True)
-    out["rsbench"] = res
+    out["rsfetch" if a.prolog else "rsbench"] = res
 if "pathtrace" in a.what:
     c = I.C4
     tris, mat, mats, cam = I.cornell_scene(c)

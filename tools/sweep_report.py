@@ -17,7 +17,8 @@ def main():
         d = json.load(open(path))
         for wl, rows in d.items():
             unit = {"mcml": "photons_per_s", "divloop": "thread_iters_per_s",
-                    "pathtrace": "paths_per_s", "rsbench": "lookups_per_s"}[wl]
+                    "pathtrace": "paths_per_s", "rsbench": "lookups_per_s",
+                    "rsfetch": "lookups_per_s"}[wl]
             base = {r["block"]: r["ms"] for r in rows if r["mode"] == "pdom"}
             print(f"## {wl} ({path.split('/')[-1]})\n")
             print("| block | mode | T | ms | speedup vs PDOM | rate | region eff | rounds | "
