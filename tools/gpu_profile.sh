@@ -20,6 +20,20 @@ timeout 1200 ncu --metrics $M --clock-control none -k regex:"divloop|commoncall|
 timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes pdom,spec --threshold 32 --unroll 1 > /dev/null 2>&1
 timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic8_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes spec --threshold 8 --unroll 1 > /dev/null 2>&1
 timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstaticu4_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes spec --threshold 32 --unroll 4 > /dev/null 2>&1
+# per-instruction SourceCounters of the simulator-validation launches (tools/region_check.py)
+SC="ncu --section SourceCounters --clock-control none"
+OL="python tools/one_launch.py"
+MCS="mcml --static --photons 131072 --iters 8"
+timeout 300 $SC -k regex:divloop -o $O/src_divloop_pdom_$TAG $OL divloop --modes pdom > /dev/null 2>&1
+timeout 300 $SC -k regex:divloop -o $O/src_divloop_spec_$TAG $OL divloop --modes spec > /dev/null 2>&1
+timeout 300 $SC -k regex:rs_ -o $O/src_rs_pdom_$TAG $OL rsbench --modes pdom > /dev/null 2>&1
+timeout 300 $SC -k regex:rs_ -o $O/src_rs_spec_$TAG $OL rsbench --modes spec > /dev/null 2>&1
+timeout 300 $SC -k regex:mcml -o $O/src_mc_pdom_$TAG $OL $MCS --modes pdom --unroll 1 > /dev/null 2>&1
+timeout 300 $SC -k regex:mcml -o $O/src_mc_spec32_$TAG $OL $MCS --modes spec --threshold 32 --unroll 1 > /dev/null 2>&1
+timeout 300 $SC -k regex:mcml -o $O/src_mc_spec8_$TAG $OL $MCS --modes spec --threshold 8 --unroll 1 > /dev/null 2>&1
+timeout 300 $SC -k regex:mcml -o $O/src_mc_spec32u4_$TAG $OL $MCS --modes spec --threshold 32 --unroll 4 > /dev/null 2>&1
+# full captures of the path tracer kernels (PDOM and the default split merge)
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:pt_ -c 2 -o $O/prof_pt_$TAG $OL pathtrace > $O/prof_pt_$TAG.log 2>&1
 # launch list of one short bench run (shares, not absolutes)
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-configs > $O/launches_$TAG.log 2>&1
 # full captures of the dominant kernel (and its PDOM baseline), at 2M photons

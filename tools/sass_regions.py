@@ -305,8 +305,10 @@ def kernel_costs(kernel_regex=".*"):
                 prev = bb_reg
         reg = {}
         unmapped = 0
+        instr = []   # (byte offset, region key or None = cold, issue weight)
         for i, x in enumerate(body):
             if i in cold:
+                instr.append((x["addr"], None, 1))
                 continue
             r = final[i]
             if r is None:
@@ -320,9 +322,13 @@ def kernel_costs(kernel_regex=".*"):
             if cm and cm.group(1) in sub_size and not x["text"].startswith("@"):
                 n += sub_size[cm.group(1)]
             reg[key] = reg.get(key, 0) + n
-        out[name] = dict(regions=reg, unmapped=unmapped, total=sum(reg.values()))
+            instr.append((x["addr"], key, n))
+        out[name] = dict(regions=reg, unmapped=unmapped, total=sum(reg.values()), instr=instr)
     return out
 
 
 if __name__ == "__main__":
-    print(json.dumps(kernel_costs(sys.argv[1] if len(sys.argv) > 1 else ".*"), indent=1))
+    res = kernel_costs(sys.argv[1] if len(sys.argv) > 1 else ".*")
+    for v in res.values():
+        v.pop("instr")
+    print(json.dumps(res, indent=1))
