@@ -122,9 +122,9 @@ __global__ void __launch_bounds__(256) rs_spec(const RsArgs a) {
   bool busy = false;                       // inside a lookup's inner loop
   uint32_t rounds = 0, rel = 0, rel_lanes = 0, adv = 0, adv_lanes = 0;
   uint32_t E_mask = __ballot_sync(kFull, !valid || a.iters == 0);  // nothing left (Cancel)
+  uint32_t P = __ballot_sync(kFull, busy);  // round ballot, re-taken at the latch
   for (;;) {
-    const uint32_t P = __ballot_sync(kFull, busy);  // @sr-region ROUND:full
-    const uint32_t R = ~(P | E_mask);
+    const uint32_t R = ~(P | E_mask);  // @sr-region ROUND:full
     if ((P | R) == 0u) break;
     if constexpr (SCHED) ++rounds;
     if ((uint32_t)__popc(P) >= a.T || R == 0u) {
@@ -153,6 +153,7 @@ __global__ void __launch_bounds__(256) rs_spec(const RsArgs a) {
       }
       E_mask = __ballot_sync(kFull, !valid || k >= a.iters);  // @sr-region ADVANCE:full
     }
+    P = __ballot_sync(kFull, busy);  // @sr-region ROUND:full
   }
   finish(a, g, valid, acc, nucs, rounds, rel, rel_lanes, adv, adv_lanes);  // @sr-region ENTRY:full
 }  // @sr-region END

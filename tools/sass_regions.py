@@ -291,10 +291,15 @@ def kernel_costs(kernel_regex=".*"):
             bbs.append((start, len(body)))
         final, prev = [None] * len(body), None
         for a_, b_ in bbs:
-            votes = {}
+            # predicated instructions are if-converted branch bodies: they say
+            # which branch they came from, not which lanes run the block, so
+            # only unpredicated instructions vote (unless there are none)
+            votes, pvotes = {}, {}
             for i in range(a_, b_):
                 if strong[i] is not None and i not in cold:
-                    votes[strong[i]] = votes.get(strong[i], 0) + 1
+                    d = pvotes if body[i]["text"].startswith("@") else votes
+                    d[strong[i]] = d.get(strong[i], 0) + 1
+            votes = votes or pvotes
             bb_reg = max(votes, key=votes.get) if votes else None
             for i in range(a_, b_):
                 # every instruction of a basic block issues with the block's
