@@ -41,3 +41,7 @@ timeout 900 ncu --set full --import-source on --clock-control none -k regex:mcml
 # dram traffic of the bench-sized dominant kernel
 timeout 600 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none -k regex:mcml_spec -c 1 --csv --log-file $O/traffic_$TAG.csv python tools/one_launch.py mcml --modes spec > /dev/null 2>&1
 ls -la $O | tail -30
+# configs[4] at N = 1: the full 10^9 photons on one GPU (3 timed steps)
+timeout 900 python bench.py --photons-per-gpu 1000000000 --steps 3 --warmup 3 --no-configs --no-cpu > $O/bench_c5_$TAG.json 2> $O/bench_c5_$TAG.err
+# CPU baselines of every config, one core and all host cores
+timeout 900 python tools/cpu_baselines.py --out $O/cpu_baselines_$TAG.json > /dev/null 2> $O/cpu_baselines_$TAG.err
