@@ -284,7 +284,8 @@ def kernel_costs(kernel_regex=".*"):
             if i > start and x["labels"]:
                 bbs.append((start, i))
                 start = i
-            if re.match(r"(@!?U?P\w+\s+)?(BRA|EXIT|RET)\b", x["text"]):
+            if re.match(r"(@!?U?P\w+\s+)?(BRA|EXIT|RET)\b", x["text"]) and \
+                    not x["text"].startswith("BRA.DIV"):
                 bbs.append((start, i + 1))
                 start = i + 1
         if start < len(body):
@@ -308,6 +309,36 @@ def kernel_costs(kernel_regex=".*"):
                 final[i] = bb_reg or strong[i] or prev or weak[i]
             if bb_reg is not None:
                 prev = bb_reg
+        # reconvergence points: the code at a BSSY's target label (and the BSYNC
+        # that waits there) runs with the mask the warp had at the BSSY -- the
+        # tail of an if/else that the compiler merged into the code after it
+        # carries the line of one arm, but it issues for every lane that
+        # entered the if, so it takes the region of the BSSY instruction
+        label_blk = {}
+        for k, (a_, b_) in enumerate(bbs):
+            for lb in body[a_]["labels"]:
+                label_blk[lb] = k
+        # (in address order: a BSSY inside a block that was itself re-assigned
+        # by an earlier reconvergence point reads its corrected region)
+        blk_start = {a_: b_ for a_, b_ in bbs}
+        open_bssy, pending = {}, {}
+        for i, x in enumerate(body):
+            if i in blk_start and i in pending:
+                for j in range(i, blk_start[i]):
+                    if not re.match(r"(?:@\S+\s+)?BSYNC", body[j]["text"]):
+                        final[j] = pending[i]
+            if i in cold:
+                continue
+            m = re.match(r"(?:@\S+\s+)?BSSY(?:\.\w+)?\s+(B\d+),\s*`\((\.L_x_\d+)\)", x["text"])
+            if m and final[i] is not None:
+                open_bssy[m.group(1)] = final[i]
+                k = label_blk.get(m.group(2))
+                if k is not None and bbs[k][0] > i:
+                    pending[bbs[k][0]] = final[i]
+                continue
+            m = re.match(r"(?:@\S+\s+)?BSYNC(?:\.\w+)?\s+(B\d+)", x["text"])
+            if m and m.group(1) in open_bssy:
+                final[i] = open_bssy[m.group(1)]
         reg = {}
         unmapped = 0
         instr = []   # (byte offset, region key or None = cold, issue weight)
