@@ -85,6 +85,10 @@ BEER_LAMBERT = MCML(layers=((1.0, 10.0, 0.0, 0.0, 0.1),), nz=100, dz=0.001)
 NO_ABSORPTION = MCML(layers=((1.4, 0.0, 50.0, 0.9, 0.02),))
 # classic MCML validation slab (n=1, mua=10, mus=90, g=0.75, d=0.02 cm)
 VAN_DE_HULST = MCML(layers=((1.0, 10.0, 90.0, 0.75, 0.02),))
+# index-mismatched absorbing slab in air, no scattering: a normally incident
+# pencil beam bounces between the two faces (Fresnel r = ((n-1)/(n+1))^2 at
+# each), so Rd, Tt and A follow the multiple-reflection series in closed form
+MISMATCHED_ABSORBER = MCML(layers=((1.4, 5.0, 0.0, 0.0, 0.1),), nz=100, dz=0.001)
 
 C1 = DivLoop()
 C2 = CommonCall()

@@ -210,7 +210,8 @@ def test_mcml_bit_exact_small(ctx, seed, flags, mode, T):
     assert_mc_equal(got, ref)
 
 
-@pytest.mark.parametrize("name", ["BEER_LAMBERT", "NO_ABSORPTION", "VAN_DE_HULST"])
+@pytest.mark.parametrize("name", ["BEER_LAMBERT", "NO_ABSORPTION", "VAN_DE_HULST",
+                                  "MISMATCHED_ABSORBER"])
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 32)])
 def test_mcml_bit_exact_pin_workloads(ctx, name, mode, T):
     m = getattr(I, name)

@@ -41,6 +41,46 @@ def test_beer_lambert_absorbed_fraction_and_depth_profile():
     assert chi2 < m.nz + 5 * math.sqrt(2 * m.nz)
 
 
+def test_mismatched_absorber_multiple_reflection_closed_form():
+    """n = 1.4 slab in air, mua = 5, mus = 0, d = 0.1 cm, pencil beam at normal
+    incidence: every boundary hit is the ca1 > COSZERO case, r = ((n-1)/(n+1))^2
+    at both faces, and (mus = 0) an interaction deposits the whole weight.  With
+    T = exp(-mua d) the photon that entered (weight w0 = 1 - r) leaves through
+    the bottom with probability T(1-r)/(1-r^2 T^2) and through the top with
+    r T^2 (1-r)/(1-r^2 T^2) (the multiple-reflection series).  Pins the
+    mismatched-boundary branch in transport: reflect vs transmit, the uz
+    reversal, s_left continuation, Rd at the top and Tt at the bottom."""
+    m = I.MISMATCHED_ABSORBER
+    p = P(m)
+    N = 400000
+    o = oracle.mcml(p, 0, N, I.PRIMARY_SEED)
+    c = o["counters"]
+    n_, mua, _, _, d = m.layers[0]
+    r = ((n_ - 1.0) / (n_ + 1.0)) ** 2
+    T = math.exp(-mua * d)
+    den = 1.0 - r * r * T * T
+    p_tt, p_rd = T * (1 - r) / den, r * T * T * (1 - r) / den
+    for k, pk in (("tt_exits", p_tt), ("rd_exits", p_rd)):
+        assert abs(c[k] / N - pk) < 5 * math.sqrt(pk * (1 - pk) / N), (k, c[k] / N, pk)
+    # every exit and every absorption carries the whole entering weight, on axis
+    w0 = np.float32(1.0) - np.float32(oracle.mcml_rsp(p))
+    fxw = int(np.float32(w0) * np.float32(FX))
+    assert int(o["Tt"].sum()) == c["tt_exits"] * fxw and int(o["Tt"][1:].sum()) == 0
+    assert int(o["Rd"].sum()) == c["rd_exits"] * fxw and int(o["Rd"][1:].sum()) == 0
+    n_abs = N - c["tt_exits"] - c["rd_exits"]
+    assert int(o["A"].sum()) == n_abs * fxw and o["A"][:, 1:].sum() == 0
+    assert c["rr_kills"] == 0 and c["capped"] == 0 and c["zero_w"] == n_abs
+    # absorption depth profile: the downward pass k contributes mua e^{-mua z}
+    # weighted by (r^2 T^2)^k, the upward pass the mirror image weighted by r T (...)
+    z = np.arange(m.nz + 1) * m.dz
+    down = np.exp(-mua * z[:-1]) - np.exp(-mua * z[1:])
+    up = np.exp(-mua * (d - z[1:])) - np.exp(-mua * (d - z[:-1]))
+    expect = N * (down + r * T * up) / den
+    counts = o["A"][:, 0] / float(fxw)
+    chi2 = ((counts - expect) ** 2 / expect).sum()
+    assert chi2 < m.nz + 5 * math.sqrt(2 * m.nz)
+
+
 def test_specular_reflectance_closed_form():
     p = P(I.C3)
     assert oracle.mcml_rsp(p) == pytest.approx(((1.0 - 1.4) / (1.0 + 1.4)) ** 2, rel=1e-6)
