@@ -28,6 +28,14 @@ LABELS_MCSTATIC8 = ["mcml_spec_static(T=8)"]
 LABELS_MCSTATICU4 = ["mcml_spec_static(T=32,U=4)"]
 
 
+def gbs(r, hbm):
+    """achieved DRAM GB/s of one launch and its share of the measured HBM peak"""
+    if not r.get("dram_bytes") or not r.get("time_ns"):
+        return "-"
+    g = r["dram_bytes"] / r["time_ns"]
+    return f"{g:.3g} ({100 * g / hbm:.2g} %)"
+
+
 def read_ncu_csv(path):
     rows = list(csv.reader(open(path)))
     hdr, data = None, {}
@@ -112,8 +120,11 @@ def main():
           "(P:234-236). `*_static` rows: the simulator-validation launches (16384 lanes x 8 "
           "photons, static assignment).", "",
           "| kernel | SIMT eff | thread-inst | warp-inst | issue active % | warps active % | "
-          "time us | DRAM bytes | L2 bytes | regs | grid x block |",
-          "|---|---|---|---|---|---|---|---|---|---|---|"]
+          "time us | DRAM bytes | DRAM GB/s (% of HBM peak) | L2 bytes | regs | grid x block |",
+          "|---|---|---|---|---|---|---|---|---|---|---|---|"]
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+    hbm = peaks.get("hbm_gbs", 6537.0)
     for lab, r in js.items():
         if lab.startswith("_"):
             continue
@@ -121,7 +132,8 @@ def main():
         md.append(f"| {lab} | {f(r['simt_efficiency'], '%.3f')} | {f(r['thread_inst'], '%.4g')} | "
                   f"{f(r['inst'], '%.4g')} | {f(r['issue_active_pct'], '%.1f')} | "
                   f"{f(r['warps_active_pct'], '%.1f')} | {f(r['time_ns'] and r['time_ns'] / 1e3, '%.1f')} | "
-                  f"{f(r['dram_bytes'], '%.3g')} | {f(r['l2_bytes'], '%.3g')} | {f(r['regs'], '%.0f')} | "
+                  f"{f(r['dram_bytes'], '%.3g')} | {gbs(r, hbm)} | "
+                  f"{f(r['l2_bytes'], '%.3g')} | {f(r['regs'], '%.0f')} | "
                   f"{f(r['grid'], '%.0f')}x{f(r['block'], '%.0f')} |")
     open(os.path.join(PROF, f"simt_{tag}.md"), "w").write("\n".join(md) + "\n")
 
