@@ -81,7 +81,7 @@ uint32_t default_block(const sr_workload& w) {
   switch (w.kind) {
     case SR_WL_DIVLOOP: return 64;
     case SR_WL_COMMONCALL: return 256;
-    case SR_WL_MCML: return 512;
+    case SR_WL_MCML: return SR_MCML_MAXT;
     case SR_WL_RSBENCH: return 256;
     default: return 128;
   }

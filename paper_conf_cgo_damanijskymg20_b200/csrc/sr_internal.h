@@ -10,6 +10,13 @@
 
 namespace sr {
 
+// MCML CTA size (and __launch_bounds__ of its kernels): 2 CTAs x 640 threads at
+// <= 48 registers (40 warps / SM) measured best on B200 (tools/exp_occ2.sh:
+// 512 -> 35.6 ms, 576 -> 34.8, 640 -> 34.8, 3 x 416 -> 35.0, 704 (spills) -> 35.7)
+#ifndef SR_MCML_MAXT
+#define SR_MCML_MAXT 640
+#endif
+
 constexpr int kCounters = 16;
 constexpr int kSchedWords = 8;  // uint32 per warp
 

@@ -7,6 +7,11 @@ from paper_conf_cgo_damanijskymg20_b200 import build as B  # noqa: E402
 
 VARIANTS = {
     "libsr_t640.so": ["SR_MCML_MAXT=640", "SR_MCML_MINB=2"],
+    "libsr_t512.so": ["SR_MCML_MAXT=512", "SR_MCML_MINB=2"],
+    "libsr_t576.so": ["SR_MCML_MAXT=576", "SR_MCML_MINB=2"],
+    "libsr_t704.so": ["SR_MCML_MAXT=704", "SR_MCML_MINB=2"],
+    "libsr_t448m3.so": ["SR_MCML_MAXT=448", "SR_MCML_MINB=3"],
+    "libsr_t416m3.so": ["SR_MCML_MAXT=416", "SR_MCML_MINB=3"],
     "libsr_t768.so": ["SR_MCML_MAXT=768", "SR_MCML_MINB=2"],
     "libsr_t1024.so": ["SR_MCML_MAXT=1024", "SR_MCML_MINB=1"],
     "libsr_t384.so": ["SR_MCML_MAXT=384", "SR_MCML_MINB=3"],
