@@ -91,6 +91,41 @@ struct Stats {
   uint32_t rays, nodes, tests;
 };
 
+// Scene reads through the read-only data path as 128-bit loads (LDG.E.128.
+// CONSTANT): a node is 4, a triangle 3, a material 2 vector loads instead of
+// one scalar load per field (the structs are 4-byte aligned, so the compiler
+// would not vectorise them itself; the image keeps every record 16-byte
+// aligned: 128-byte header, 64-byte nodes, 48-byte triangles).
+__device__ __forceinline__ PtNode load_node(const PtNode* base, int32_t i) {
+  const float4* q = reinterpret_cast<const float4*>(base + i);
+  const float4 x = __ldg(q), y = __ldg(q + 1), z = __ldg(q + 2);
+  const int4 w = __ldg(reinterpret_cast<const int4*>(q + 3));
+  PtNode n;
+  n.b0lo[0] = x.x; n.b0lo[1] = x.y; n.b0lo[2] = x.z; n.b0hi[0] = x.w;
+  n.b0hi[1] = y.x; n.b0hi[2] = y.y; n.b1lo[0] = y.z; n.b1lo[1] = y.w;
+  n.b1lo[2] = z.x; n.b1hi[0] = z.y; n.b1hi[1] = z.z; n.b1hi[2] = z.w;
+  n.ref0 = w.x; n.cnt0 = w.y; n.ref1 = w.z; n.cnt1 = w.w;
+  return n;
+}
+__device__ __forceinline__ PtTri load_tri(const PtTri* base, int32_t i) {
+  const float4* q = reinterpret_cast<const float4*>(base + i);
+  const float4 x = __ldg(q), y = __ldg(q + 1);
+  const uint4 z = __ldg(reinterpret_cast<const uint4*>(q + 2));
+  PtTri t;
+  t.v0[0] = x.x; t.v0[1] = x.y; t.v0[2] = x.z; t.e1[0] = x.w;
+  t.e1[1] = y.x; t.e1[2] = y.y; t.e2[0] = y.z; t.e2[1] = y.w;
+  t.e2[2] = __uint_as_float(z.x); t.id = z.y; t.mat = z.z; t.pad = z.w;
+  return t;
+}
+__device__ __forceinline__ PtMat load_mat(const PtMat* base, uint32_t i) {
+  const float4* q = reinterpret_cast<const float4*>(base + i);
+  const float4 x = __ldg(q), y = __ldg(q + 1);
+  PtMat m;
+  m.kind = x.x; m.r = x.y; m.g = x.z; m.b = x.w;
+  m.er = y.x; m.eg = y.y; m.eb = y.z; m.ior = y.w;
+  return m;
+}
+
 // Conservative slab test against a padded box: accept when the ray's
 // parametric interval [tmin, tbest] can touch the box (slack 1e-5 relative).
 __device__ __forceinline__ bool box_hit(const float* lo, const float* hi, V3 o, V3 inv, float tb,
@@ -177,7 +212,7 @@ __device__ __forceinline__ void trav_begin(Trav& tr, V3 o, V3 d) {
 
 // returns false when the traversal is finished
 __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) {
-  const PtNode N = a.nodes[tr.node];
+  const PtNode N = load_node(a.nodes, tr.node);
   ++st.nodes;
   float tn0, tn1;
   const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, tr.o, tr.inv, tr.tb, tn0);
@@ -186,7 +221,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
   if (h0 && N.cnt0 > 0) {
     for (int32_t k = 0; k < N.cnt0; ++k) {
       const int64_t before = tr.ib;
-      tri_test(a.tris[N.ref0 + k], tr.o, tr.d, tr.tb, tr.ib, tr.mb);
+      tri_test(load_tri(a.tris, N.ref0 + k), tr.o, tr.d, tr.tb, tr.ib, tr.mb);
       if (tr.ib != before) tr.slot = (uint32_t)(N.ref0 + k);
       ++st.tests;
     }
@@ -194,7 +229,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
   if (h1 && N.cnt1 > 0) {
     for (int32_t k = 0; k < N.cnt1; ++k) {
       const int64_t before = tr.ib;
-      tri_test(a.tris[N.ref1 + k], tr.o, tr.d, tr.tb, tr.ib, tr.mb);
+      tri_test(load_tri(a.tris, N.ref1 + k), tr.o, tr.d, tr.tb, tr.ib, tr.mb);
       if (tr.ib != before) tr.slot = (uint32_t)(N.ref1 + k);
       ++st.tests;
     }
@@ -225,7 +260,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
 // trav_leaf tests ONE queued triangle.  Returns: a leaf triangle is pending
 // (na > 0), else a node is pending (node >= 0), else the traversal is done.
 __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, Stats& st) {
-  const PtNode N = a.nodes[tr.node];
+  const PtNode N = load_node(a.nodes, tr.node);
   ++st.nodes;
   float tn0, tn1;
   const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, tr.o, tr.inv, tr.tb, tn0);
@@ -252,7 +287,7 @@ __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, Stats& st) 
 
 __device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, Stats& st) {
   const int64_t before = tr.ib;
-  tri_test(a.tris[tr.la], tr.o, tr.d, tr.tb, tr.ib, tr.mb);
+  tri_test(load_tri(a.tris, tr.la), tr.o, tr.d, tr.tb, tr.ib, tr.mb);
   if (tr.ib != before) tr.slot = (uint32_t)tr.la;
   ++st.tests;
   ++tr.la;
@@ -314,13 +349,13 @@ __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
   const uint32_t mat = tr.mb, slot = tr.slot;
   bool end = hit < 0;
   if (!end) {
-    const PtMat m = a.mats[mat];
+    const PtMat m = load_mat(a.mats, mat);
     const uint32_t kind = (uint32_t)m.kind;
     p.rad = add(p.rad, mk(p.thr.x * m.er, p.thr.y * m.eg, p.thr.z * m.eb));
     if (kind == 3u) {
       end = true;
     } else {
-      const PtTri& T = a.tris[slot];
+      const PtTri T = load_tri(a.tris, (int32_t)slot);
       const V3 e1 = mk(T.e1[0], T.e1[1], T.e1[2]);
       const V3 e2 = mk(T.e2[0], T.e2[1], T.e2[2]);
       const V3 ng = normalize(cross(e1, e2));
