@@ -481,9 +481,10 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
     w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth)
     ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
     res = {"scene_triangles": int(len(tris)), "scene_bytes": int(used)}
-    # node-granularity Loop Merge, 8 node visits per release, soft barrier T = 8
-    # (best of the tools/sweep.py threshold sweep, profiles/threshold_sweep_*.md)
-    for name, mode, thr in (("pdom", sr.PDOM, 0), ("spec_t8", sr.SPEC_LOOP, 8)):
+    # split node-granularity Loop Merge, 8 node visits per release, soft barrier
+    # T = inputs.C4.threshold (best of the threshold sweep, profiles/)
+    sname = f"spec_t{c.threshold}"
+    for name, mode, thr in (("pdom", sr.PDOM, 0), (sname, sr.SPEC_LOOP, c.threshold)):
         ms = timer.time_steps(lambda: sr.sr_run(w, c.n_pixels, c.spp, I.PRIMARY_SEED, mode, thr),
                               max(3, min(args.steps, 5)), 1)
         t = statistics.median(ms)
@@ -491,7 +492,7 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
         res[name] = {"value": c.n_pixels * c.spp / (t * 1e-3), "unit": "paths/s", "ms": t,
                      "rays": int(cnt[1]), "node_visits": int(cnt[2]), "tri_tests": int(cnt[3]),
                      "launch": sr.sr_last_launch()}
-    res["speedup_vs_pdom"] = res["spec_t8"]["value"] / res["pdom"]["value"]
+    res["speedup_vs_pdom"] = res[sname]["value"] / res["pdom"]["value"]
     out["pathtrace"] = res
     return out
 

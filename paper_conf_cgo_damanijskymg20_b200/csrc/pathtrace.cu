@@ -42,14 +42,15 @@ constexpr float kDetEps = 1.0e-12f;
 // dynamic shared memory (23 for configs[3]); kMaxStack bounds what a scene may need
 constexpr uint32_t kMaxStack = 256;
 // CTAs of 128 threads per SM the register budget must allow, per kernel, each
-// at its best measured setting (profiles/pt_tuning_r01.md): the latency-bound
-// PDOM kernel wants 8 (64 registers), the merged kernels 6 (80 registers).
+// at its best measured setting (profiles/pt_tuning_r01.md): both latency-bound
+// kernels want 8 (64 registers; the merged kernel spills 32 bytes and is still
+// faster than at 6 CTAs / 80 registers: 37.3 vs 41.1 ms at T = 12).
 // (An L1 prefetch of the next node / triangle was measured 5 % slower.)
 #ifndef SR_PT_MINB_PDOM
 #define SR_PT_MINB_PDOM 8
 #endif
 #ifndef SR_PT_MINB_SPEC
-#define SR_PT_MINB_SPEC 6
+#define SR_PT_MINB_SPEC 8
 #endif
 
 struct V3 {
@@ -141,8 +142,8 @@ __device__ __forceinline__ bool box_hit(const float* lo, const float* hi, V3 o, 
 
 // Moller-Trumbore exactly as the oracle (e1, e2 precomputed with the same
 // binary32 subtractions).
-__device__ __forceinline__ void tri_test(const PtTri& T, V3 o, V3 d, float& tb, int64_t& ib,
-                                         uint32_t& mb) {
+__device__ __forceinline__ void tri_test(const PtTri& T, int32_t at, V3 o, V3 d, float& tb,
+                                         int32_t& ib, uint32_t& mb, uint32_t& slot) {
   const V3 v0 = mk(T.v0[0], T.v0[1], T.v0[2]);
   const V3 e1 = mk(T.e1[0], T.e1[1], T.e1[2]);
   const V3 e2 = mk(T.e2[0], T.e2[1], T.e2[2]);
@@ -158,11 +159,12 @@ __device__ __forceinline__ void tri_test(const PtTri& T, V3 o, V3 d, float& tb, 
   if (v < 0.0f || u + v > 1.0f) return;
   const float t = dot(e2, qv) * inv;
   if (!(t > kTmin)) return;
-  const int64_t id = (int64_t)T.id;
+  const int32_t id = (int32_t)T.id;        // < 2^31 (sr_scene_build checks)
   if (t < tb || (t == tb && id < ib)) {   // ties -> smaller original id (= brute force)
     tb = t;
     ib = id;
     mb = T.mat;
+    slot = (uint32_t)at;
   }
 }
 
@@ -178,22 +180,21 @@ __device__ __forceinline__ void tri_test(const PtTri& T, V3 o, V3 d, float& tb, 
 struct Trav {
   V3 o, d, inv;
   float tb;
-  int64_t ib;
+  int32_t ib;       // original index of the closest triangle so far (-1: none)
   uint32_t mb, slot;
   int32_t node;
   int32_t sp;
-  int32_t* stk;     // this thread's column of the CTA's shared stack
-  uint32_t stride;  // blockDim.x
   // split merge (default): leaf ranges found by the last node visit, tested later by
   // trav_leaf (current range la/na, queued range lb/nb)
   int32_t la, lb;
   uint32_t na, nb;
 };
 
-__device__ __forceinline__ void trav_bind(Trav& tr) {
-  extern __shared__ int32_t pt_stack_smem[];
-  tr.stk = pt_stack_smem + threadIdx.x;
-  tr.stride = blockDim.x;
+extern __shared__ int32_t pt_stack_smem[];
+// entry i of this thread's stack column (addressed from threadIdx / blockDim,
+// so no per-lane pointer is kept in registers)
+__device__ __forceinline__ int32_t& stk(int32_t i) {
+  return pt_stack_smem[(uint32_t)i * blockDim.x + threadIdx.x];
 }
 
 __device__ __forceinline__ void trav_begin(Trav& tr, V3 o, V3 d) {
@@ -220,17 +221,13 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
   // leaves: test their triangles now; inner children: descend / push
   if (h0 && N.cnt0 > 0) {
     for (int32_t k = 0; k < N.cnt0; ++k) {
-      const int64_t before = tr.ib;
-      tri_test(load_tri(a.tris, N.ref0 + k), tr.o, tr.d, tr.tb, tr.ib, tr.mb);
-      if (tr.ib != before) tr.slot = (uint32_t)(N.ref0 + k);
+      tri_test(load_tri(a.tris, N.ref0 + k), N.ref0 + k, tr.o, tr.d, tr.tb, tr.ib, tr.mb, tr.slot);
       ++st.tests;
     }
   }
   if (h1 && N.cnt1 > 0) {
     for (int32_t k = 0; k < N.cnt1; ++k) {
-      const int64_t before = tr.ib;
-      tri_test(load_tri(a.tris, N.ref1 + k), tr.o, tr.d, tr.tb, tr.ib, tr.mb);
-      if (tr.ib != before) tr.slot = (uint32_t)(N.ref1 + k);
+      tri_test(load_tri(a.tris, N.ref1 + k), N.ref1 + k, tr.o, tr.d, tr.tb, tr.ib, tr.mb, tr.slot);
       ++st.tests;
     }
   }
@@ -239,7 +236,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
   if (in0 && in1) {
     const bool first0 = tn0 <= tn1;
     next = first0 ? N.ref0 : N.ref1;
-    if ((uint32_t)tr.sp < a.stack_cap) tr.stk[(tr.sp++) * tr.stride] = first0 ? N.ref1 : N.ref0;
+    if ((uint32_t)tr.sp < a.stack_cap) stk(tr.sp++) = first0 ? N.ref1 : N.ref0;
   } else if (in0) {
     next = N.ref0;
   } else if (in1) {
@@ -247,7 +244,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
   }
   if (next < 0) {
     if (tr.sp == 0) return false;
-    next = tr.stk[(--tr.sp) * tr.stride];
+    next = stk(--tr.sp);
   }
   tr.node = next;
   return true;
@@ -275,20 +272,18 @@ __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, Stats& st) 
   if (in0 && in1) {
     const bool first0 = tn0 <= tn1;
     next = first0 ? N.ref0 : N.ref1;
-    if ((uint32_t)tr.sp < a.stack_cap) tr.stk[(tr.sp++) * tr.stride] = first0 ? N.ref1 : N.ref0;
+    if ((uint32_t)tr.sp < a.stack_cap) stk(tr.sp++) = first0 ? N.ref1 : N.ref0;
   } else if (in0) {
     next = N.ref0;
   } else if (in1) {
     next = N.ref1;
   }
-  if (next < 0 && tr.sp > 0) next = tr.stk[(--tr.sp) * tr.stride];
+  if (next < 0 && tr.sp > 0) next = stk(--tr.sp);
   tr.node = next;
 }
 
 __device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, Stats& st) {
-  const int64_t before = tr.ib;
-  tri_test(load_tri(a.tris, tr.la), tr.o, tr.d, tr.tb, tr.ib, tr.mb);
-  if (tr.ib != before) tr.slot = (uint32_t)tr.la;
+  tri_test(load_tri(a.tris, tr.la), tr.la, tr.o, tr.d, tr.tb, tr.ib, tr.mb, tr.slot);
   ++st.tests;
   ++tr.la;
   if (--tr.na == 0u) {
@@ -302,7 +297,7 @@ __device__ __forceinline__ int64_t closest_hit(const PtArgs& a, Trav& tr, V3 o, 
   trav_begin(tr, o, d);
   while (trav_step(a, tr, st)) {
   }
-  return tr.ib;
+  return (int64_t)tr.ib;
 }
 
 struct Path {
@@ -449,7 +444,6 @@ __global__ void __launch_bounds__(128, SR_PT_MINB_PDOM) pt_pdom(const PtArgs a) 
   p.sum = mk(0.0f, 0.0f, 0.0f);
   p.alive = false;
   Trav tr;
-  trav_bind(tr);
   Stats st{0, 0, 0};
   uint32_t paths = 0, outer = 0, rel = 0, rel_lanes = 0, launch_lanes = 0;
   for (uint32_t s = 0; s < a.spp; ++s) {
@@ -491,7 +485,6 @@ __global__ void __launch_bounds__(128, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) 
   p.alive = false;
   p.s = 0;
   Trav tr;
-  trav_bind(tr);
   bool trav = false;                   // NODE: a ray of this lane is being traversed
   Stats st{0, 0, 0};
   uint32_t paths = 0, rounds = 0, rel = 0, rel_lanes = 0, adv = 0, adv_lanes = 0;
@@ -584,7 +577,6 @@ __global__ void pt_query(const PtArgs a) {
   const float* r = a.q_rays + 6 * i;
   Stats st{0, 0, 0};
   Trav tr;
-  trav_bind(tr);
   const int64_t h = closest_hit(a, tr, mk(r[0], r[1], r[2]), mk(r[3], r[4], r[5]), st);
   a.q_hit[i] = h;
   a.q_t[i] = tr.tb;

@@ -112,7 +112,7 @@ class PathTrace:
     subdiv: int = 5          # 20 * 4^5 = 20480 triangles per sphere; 51 -> 1,044,494 total
     fov_deg: float = 65.0
     scene_seed: int = 20200222
-    threshold: int = 32
+    threshold: int = 12      # best of the tools/exp_pt_minb.sh sweep (split merge, unroll 8)
 
     @property
     def n_pixels(self) -> int:

@@ -17,6 +17,7 @@ VARIANTS = {
     "libsr_t384.so": ["SR_MCML_MAXT=384", "SR_MCML_MINB=3"],
     "libsr_pts5.so": ["SR_PT_MINB_SPEC=5"],
     "libsr_pts7.so": ["SR_PT_MINB_SPEC=7"],
+    "libsr_pts8.so": ["SR_PT_MINB_SPEC=8"],
     "libsr_ptp6.so": ["SR_PT_MINB_PDOM=6"],
 }
 if __name__ == "__main__":

@@ -67,7 +67,7 @@ if "pathtrace" in a.what:
     ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
     for md in modes:
         sr.sr_run(w, c.n_pixels, c.spp, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
-                  0 if md == "pdom" else 8)   # the path tracer's best threshold
+                  0 if md == "pdom" else c.threshold)   # the path tracer's best threshold
 torch.cuda.synchronize()
 sr.sr_finalize()
 print("ok")

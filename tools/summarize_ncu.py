@@ -22,7 +22,7 @@ PROF = os.path.join(ROOT, "profiles")
 # launch order of tools/one_launch.py (default: every family, pdom then spec)
 LABELS_ALL = ["divloop_pdom", "divloop_spec(T=16)", "commoncall_pdom", "commoncall_spec",
               "mcml_pdom", "mcml_spec(T=32)", "rs_pdom", "rs_spec(T=24)", "pt_pdom",
-              "pt_spec(T=8)"]
+              "pt_spec(T=12)"]
 LABELS_MCSTATIC = ["mcml_pdom_static", "mcml_spec_static(T=32)"]
 LABELS_MCSTATIC8 = ["mcml_spec_static(T=8)"]
 LABELS_MCSTATICU4 = ["mcml_spec_static(T=32,U=4)"]
