@@ -299,6 +299,19 @@ def main():
         return float(t.item())
 
     t_spec = max_over_ranks(statistics.mean(ms_spec))
+
+    # the step's one collective timed alone (N > 1): the tally all-reduce over
+    # GRID+COUNTERS, CUDA events on the launching stream, max over ranks -- the
+    # measurement behind DESIGN.md's NEXT-4 decision (fusing it into the kernel
+    # tail cannot move a step it is this small a share of)
+    coll = None
+    if ws_n > 1:
+        def allreduce_only():
+            P.allreduce_tallies(tallies, stream=stream)
+        ms_ar = timer.time_steps(allreduce_only, args.steps, args.warmup, barrier)
+        t_ar = max_over_ranks(statistics.mean(ms_ar))
+        coll = {"op": f"all_reduce(SUM) int64, {args.dist_backend}", "bytes": tb + cb,
+                "ms": t_ar, "share_of_step": t_ar / t_spec}
     t_pdom = max_over_ranks(statistics.mean(ms_pdom))
     total = per_rank * ws_n
     value = total / (t_spec * 1e-3)
@@ -383,6 +396,7 @@ def main():
                     "d2h_bytes_per_step": tb + cb},
             "gpu_launches": args.steps,
             "roofline": rl,
+            "collective": coll,
         }
         simt = load_json(os.path.join(ROOT, "profiles", "simt_efficiency.json"))
         if simt:

@@ -34,6 +34,7 @@ def test_bench_single_gpu_contract():
     assert d["n_gpus"] == 1 and d["value"] > 0 and d["speedup_vs_pdom"] > 1.0
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert d["gpu_launches"] == 3
+    assert d["collective"] is None   # no collective at N = 1
 
 
 def test_bench_two_rank_path_gloo():
@@ -50,6 +51,8 @@ def test_bench_two_rank_path_gloo():
     assert d["n_gpus"] == 2 and d["scaling"] == "weak"
     assert d["config"]["photons_per_gpu"] == 512000   # a multiple of photons_per_lane
     assert "cpu_baseline" not in d and "configs" not in d   # rank 0 at N=1 only
+    c = d["collective"]   # the tally all-reduce timed alone
+    assert c["ms"] > 0 and c["bytes"] > 0 and c["share_of_step"] > 0
 
 
 def test_bench_reference_arm():
