@@ -356,6 +356,25 @@ def main():
     eff_spec = region_eff(sr.SPEC_LOOP, T)
     eff_pdom = region_eff(sr.PDOM, 0)
 
+    # N > 1: the whole job's photons once more on rank 0 in ONE launch (ids
+    # [0, N x per_rank), the union of the shards) -- the all-reduced tallies of
+    # the last step must equal it bit for bit (SURVEY.md Sec. 8(e) invariant)
+    same_as_one_gpu = None
+    if ws_n > 1:
+        if rank == 0:
+            w_all = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz,
+                                     m.step_cap, task_offset=P.task_offset_of(0, per_rank),
+                                     block=args.block,
+                                     unroll=args.unroll if args.unroll else m.merge_unroll)
+            nt_all = nt * ws_n
+            ctx.ensure(sr.sr_workspace_bytes(w_all, nt_all))
+            sr.sr_run(w_all, nt_all, iters, I.PRIMARY_SEED, sr.SPEC_LOOP, T)
+            ref = torch.empty(tb + cb, dtype=torch.uint8, pin_memory=True)
+            sr.sr_tally(sr.T_GRID, ref.data_ptr(), tb)
+            sr.sr_tally(sr.T_COUNTERS, ref.data_ptr() + tb, cb)
+            same_as_one_gpu = bool(torch.equal(ref, host))
+        dist.barrier()
+
     peaks = load_json(PEAKS_FILE) or {}
     consts = load_json(PROFILE_CONST) or {}
     clocks = clk.summary()
@@ -397,6 +416,7 @@ def main():
             "gpu_launches": args.steps,
             "roofline": rl,
             "collective": coll,
+            "tallies_equal_single_gpu_run": same_as_one_gpu,
         }
         simt = load_json(os.path.join(ROOT, "profiles", "simt_efficiency.json"))
         if simt:

@@ -53,6 +53,7 @@ def test_bench_two_rank_path_gloo():
     assert "cpu_baseline" not in d and "configs" not in d   # rank 0 at N=1 only
     c = d["collective"]   # the tally all-reduce timed alone
     assert c["ms"] > 0 and c["bytes"] > 0 and c["share_of_step"] > 0
+    assert d["tallies_equal_single_gpu_run"] is True   # sharded + all-reduced == one launch
 
 
 def test_bench_reference_arm():
