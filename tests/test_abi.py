@@ -161,3 +161,11 @@ def test_sass_is_sm100a_and_uses_the_intended_instructions():
             assert ops(r"\bVOTE\.", f) >= 2, f          # __ballot_sync scheduler
         if "ILi125ELb0" in f:
             assert ops(r"\bFFMA2\b", f) == 500, f       # 1000 FMAs as FFMA2, unrolled
+        if "mcml_" in f:
+            # paired IEEE products only: every FFMA2 adds the -0 pair from the kernel
+            # parameters (a uniform register), never a contracted product + sum
+            ff = [l for l in funcs[f] if re.search(r"\bFFMA2\b", l)]
+            assert ff, f
+            for l in ff:
+                addend = re.search(r"FFMA2\s+[^;]*,\s*([^,;]+);", l).group(1)
+                assert addend.strip().startswith("UR"), (f, l)
