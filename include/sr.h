@@ -212,6 +212,23 @@ enum { SR_FN_LOGF = 0, SR_FN_SIN2PI = 1, SR_FN_COS2PI = 2, SR_FN_EXPENSIVE_1000 
        SR_FN_EXPENSIVE_2000 = 4 };
 SR_API int sr_math_eval(int fn, const float* x_dev, float* out_dev, uint64_t n);
 
+/* Diagnostics: the MC step's IEEE divisions and square roots on their known
+ * operand domains (nvcc's fast path without the FCHK range
+ * check and slow-path branch), out[i] = fn(p, x[i]), on the context stream
+ * (no synchronize).  x_dev, out_dev: device arrays of n floats, caller-owned.
+ *   SR_FNP_DIV_XP    x / p             (div_dom)
+ *   SR_FNP_DIV_PX    p / x             (div_dom)
+ *   SR_FNP_SQRT      sqrt(x)           (sqrt_dom, p unused)
+ *   SR_FNP_HG_COST   Henyey-Greenstein cos(theta) for g = p, xi = x (R6)
+ *   SR_FNP_HG_SINT   sqrt(1 - cos(theta)^2) of the same
+ * Each equals the IEEE binary32 result bit for bit on the domain its call
+ * site guarantees; outside it the result is unspecified.
+ * Errors: SR_E_STATE before sr_init; SR_E_INVALID (unknown fn, NULL with
+ * n > 0); SR_E_CUDA. */
+enum { SR_FNP_DIV_XP = 0, SR_FNP_DIV_PX = 1, SR_FNP_SQRT = 2, SR_FNP_HG_COST = 3,
+       SR_FNP_HG_SINT = 4 };
+SR_API int sr_math_eval_p(int fn, float p, const float* x_dev, float* out_dev, uint64_t n);
+
 /* Diagnostics: closest hit of n rays against a scene built by sr_scene_build,
  * with the BVH traversal the PATHTRACE kernels use (reading R7).
  *   rays_dev  device, n x 6 floats {origin xyz, direction xyz}

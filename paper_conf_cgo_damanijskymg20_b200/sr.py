@@ -27,9 +27,10 @@ MC_COUNTERS = ["photons", "steps", "rd_exits", "tt_exits", "rr_kills", "rr_survi
                "zero_w"]
 EXPORTS = ["sr_init", "sr_workspace_bytes", "sr_workspace_region", "sr_run", "sr_tally",
            "sr_finalize", "sr_last_error", "sr_build_info", "sr_last_launch", "sr_math_eval",
-           "sr_pt_closest", "sr_scene_build", "sr_scene_build_host"]
+           "sr_math_eval_p", "sr_pt_closest", "sr_scene_build", "sr_scene_build_host"]
 PT_COUNTERS = ["paths", "rays", "node_visits", "tri_tests"]
 FN_LOGF, FN_SIN2PI, FN_COS2PI, FN_EXPENSIVE_1000, FN_EXPENSIVE_2000 = 0, 1, 2, 3, 4
+FNP_DIV_XP, FNP_DIV_PX, FNP_SQRT, FNP_HG_COST, FNP_HG_SINT = 0, 1, 2, 3, 4
 
 
 class SRError(RuntimeError):
@@ -103,6 +104,8 @@ def load(path: str | None = None):
     L.sr_last_launch.argtypes = [C.POINTER(C.c_uint32)]
     L.sr_math_eval.argtypes = [C.c_int, vp, vp, u64]
     L.sr_math_eval.restype = C.c_int
+    L.sr_math_eval_p.argtypes = [C.c_int, C.c_float, vp, vp, u64]
+    L.sr_math_eval_p.restype = C.c_int
     L.sr_pt_closest.argtypes = [vp, vp, vp, vp, u64]
     L.sr_pt_closest.restype = C.c_int
     fp, up = C.POINTER(C.c_float), C.POINTER(C.c_uint32)
@@ -160,6 +163,10 @@ def sr_build_info() -> str:
 
 def sr_math_eval(fn: int, x_ptr: int, out_ptr: int, n: int) -> None:
     _check(load().sr_math_eval(fn, x_ptr, out_ptr, n))
+
+
+def sr_math_eval_p(fn: int, p: float, x_ptr: int, out_ptr: int, n: int) -> None:
+    _check(load().sr_math_eval_p(fn, p, x_ptr, out_ptr, n))
 
 
 def sr_pt_closest(scene_ptr: int, rays_ptr: int, hit_ptr: int, t_ptr: int, n: int) -> None:

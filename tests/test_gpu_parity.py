@@ -68,6 +68,95 @@ def test_device_expensive_bit_exact(ctx, fn):
     assert np.array_equal(od.cpu().numpy().view(np.uint32), oracle.eval_batch(fn, x).view(np.uint32))
 
 
+# ---------------------------- the MC step's division / sqrt on their domains
+def eval_p(ctx, fn, p, x):
+    xd = torch.from_numpy(np.ascontiguousarray(x, np.float32)).cuda()
+    od = torch.empty_like(xd)
+    sr.sr_math_eval_p(fn, float(np.float32(p)), xd.data_ptr(), od.data_ptr(), x.size)
+    ctx.stream.synchronize()
+    return od.cpu().numpy()
+
+
+def assert_bits(got, ref, x):
+    bad = np.nonzero(got.view(np.uint32) != ref.view(np.uint32))[0]
+    assert bad.size == 0, (bad.size, x[bad[:5]], got[bad[:5]], ref[bad[:5]])
+
+
+F32 = np.float32
+ALL_XI = (np.arange(1 << 24, dtype=np.float64) * 2.0**-24).astype(F32)   # every U01 value
+
+
+@pytest.mark.parametrize("mut", [100.0, 200.0, 2.0**-20, 2.0**20, 7.31, 1000.0])
+def test_div_dom_path_length_every_rng_input(ctx, mut):
+    """s = -log(U01c)/mu_t: the kernel's div_dom(log, mu_t) negated == IEEE (-log)/mu_t on
+    all 2^24 inputs (IEEE division is sign-symmetric, the numerator is never -0)."""
+    x = ((np.arange(1 << 24, dtype=np.float64) + 1) * 2.0**-24).astype(F32)
+    lg = oracle.eval_batch(sr.FN_LOGF, x)
+    got = -eval_p(ctx, sr.FNP_DIV_XP, mut, lg)
+    assert_bits(got, (-lg) / F32(mut), lg)
+
+
+@pytest.mark.parametrize("p", [3.0, -0.37, 2.0**-40, 2.0**40, 1.0 + 2.0**-23])
+def test_div_dom_log_uniform_operands(ctx, p):
+    """x / p and p / x for 2^22 operands of both signs, log-uniform over [2^-60, 2^60]."""
+    rng = np.random.default_rng(7)
+    n = 1 << 22
+    x = (np.exp2(rng.uniform(-60, 60, n)) * rng.choice([-1.0, 1.0], n)).astype(F32)
+    x[:3] = [F32(1.0), F32(-1.0), F32(0.0)]   # +0 / p is in the domain for p > 0 only
+    pf = F32(p)
+    with np.errstate(divide="ignore"):
+        got = eval_p(ctx, sr.FNP_DIV_XP, pf, x)
+        ref = x / pf
+        keep = (x != 0) | (pf > 0)
+        assert_bits(got[keep], ref[keep], x[keep])
+        got = eval_p(ctx, sr.FNP_DIV_PX, pf, x[3:])
+        assert_bits(got, pf / x[3:], x[3:])
+
+
+def test_sqrt_dom_matches_ieee(ctx):
+    """every binary32 in [2^-25, 1) (the 1 - c^2 arguments), +0, and 2^22 log-uniform
+    values over [2^-101, 2^127]"""
+    rng = np.random.default_rng(3)
+    dense = np.arange(np.float32(2.0**-25).view(np.uint32), np.float32(1.0).view(np.uint32),
+                      dtype=np.uint32).view(F32)
+    wide = np.exp2(rng.uniform(-101, 127, 1 << 22)).astype(F32)
+    x = np.concatenate([dense, wide, np.array([0.0, 1.0, 2.0**-101], F32)])
+    assert_bits(eval_p(ctx, sr.FNP_SQRT, 0.0, x), np.sqrt(x), x)
+
+
+def hg_ieee(g, xi):
+    """oracle/mcml.c's Henyey-Greenstein cos(theta) (reading R6), binary32 step by step"""
+    g = F32(g)
+    g2 = g * g
+    one_m_g2, one_p_g2, one_m_g, two_g = F32(1) - g2, F32(1) + g2, F32(1) - g, F32(2) * g
+    tmp = one_m_g2 / (one_m_g + two_g * xi)
+    cost = (one_p_g2 - tmp * tmp) / two_g
+    return np.clip(cost, F32(-1), F32(1)).astype(F32)
+
+
+@pytest.mark.parametrize("g", [0.80, 0.90, 0.75, -0.8, 0.5, -0.3, 2.0**-18, -(2.0**-18),
+                               0.99999994])
+def test_hg_cost_and_sint_every_rng_input(ctx, g):
+    """the MC step's HG cos(theta) and sin(theta) on all 2^24 xi == IEEE binary32"""
+    cost = hg_ieee(g, ALL_XI)
+    assert_bits(eval_p(ctx, sr.FNP_HG_COST, g, ALL_XI), cost, ALL_XI)
+    assert_bits(eval_p(ctx, sr.FNP_HG_SINT, g, ALL_XI), np.sqrt(F32(1) - cost * cost), ALL_XI)
+
+
+@pytest.mark.parametrize("layers", [
+    ((1.4, 4.0, 96.0, 1e-30, 0.01), (1.4, 1.0, 199.0, 0.9, 0.1)),   # |g| < 2^-18
+    ((1.3, 2e-7, 1e-7, 0.5, 0.05),),                                   # mu_t < 2^-20
+    ((1.3, 2e6, 1e6, 0.5, 0.05),),                                     # mu_t > 2^20
+])
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 32)])
+def test_mcml_outside_fast_domain_bit_exact(ctx, layers, mode, T):
+    """layers outside the fast division domain run the guarded-IEEE kernels: still exact"""
+    m = I.MCML(layers=layers)
+    ref = mc_oracle(m, 0, 2048, 5)
+    got = run_mc(ctx, mc_workload(m), 256, 8, 5, mode, T, m)
+    assert_mc_equal(got, ref)
+
+
 # ------------------------------------------------------------------ config 1
 @pytest.mark.parametrize("seed", SEEDS)
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 4),
