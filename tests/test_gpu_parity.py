@@ -143,15 +143,16 @@ def test_hg_cost_and_sint_every_rng_input(ctx, g):
     assert_bits(eval_p(ctx, sr.FNP_HG_SINT, g, ALL_XI), np.sqrt(F32(1) - cost * cost), ALL_XI)
 
 
-@pytest.mark.parametrize("layers", [
-    ((1.4, 4.0, 96.0, 1e-30, 0.01), (1.4, 1.0, 199.0, 0.9, 0.1)),   # |g| < 2^-18
-    ((1.3, 2e-7, 1e-7, 0.5, 0.05),),                                   # mu_t < 2^-20
-    ((1.3, 2e6, 1e6, 0.5, 0.05),),                                     # mu_t > 2^20
+@pytest.mark.parametrize("layers,dr", [
+    (((1.4, 4.0, 96.0, 1e-30, 0.01), (1.4, 1.0, 199.0, 0.9, 0.1)), 0.01),   # |g| < 2^-18
+    (((1.3, 2e-7, 1e-7, 0.5, 0.05),), 0.01),                                 # mu_t < 2^-20
+    (((1.3, 2e6, 1e6, 0.5, 0.05),), 0.01),                                   # mu_t > 2^20
+    (I.THREE_LAYER, 1e-13),                                                  # dr < 2^-40
 ])
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 32)])
-def test_mcml_outside_fast_domain_bit_exact(ctx, layers, mode, T):
+def test_mcml_outside_fast_domain_bit_exact(ctx, layers, dr, mode, T):
     """layers outside the fast division domain run the guarded-IEEE kernels: still exact"""
-    m = I.MCML(layers=layers)
+    m = I.MCML(layers=layers, dr=dr)
     ref = mc_oracle(m, 0, 2048, 5)
     got = run_mc(ctx, mc_workload(m), 256, 8, 5, mode, T, m)
     assert_mc_equal(got, ref)
