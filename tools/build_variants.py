@@ -15,6 +15,8 @@ VARIANTS = {
     "libsr_t768.so": ["SR_MCML_MAXT=768", "SR_MCML_MINB=2"],
     "libsr_t1024.so": ["SR_MCML_MAXT=1024", "SR_MCML_MINB=1"],
     "libsr_t384.so": ["SR_MCML_MAXT=384", "SR_MCML_MINB=3"],
+    "libsr_t512m3.so": ["SR_MCML_MAXT=512", "SR_MCML_MINB=3"],
+    "libsr_t480m3.so": ["SR_MCML_MAXT=480", "SR_MCML_MINB=3"],
     "libsr_pts5.so": ["SR_PT_MINB_SPEC=5"],
     "libsr_pts7.so": ["SR_PT_MINB_SPEC=7"],
     "libsr_pts8.so": ["SR_PT_MINB_SPEC=8"],

@@ -75,14 +75,15 @@ def marked_call_lines(path):
     while changed:
         changed = False
         for f, lines in body.items():
-            if f not in marked and any(re.search(r"\b%s\s*\(" % g, c)
+            if f not in marked and any(re.search(r"\b%s\s*(?:<[^<>()]*>)?\s*\(" % g, c)
                                        for g in marked for c in lines[1:]):
                 marked.add(f)
                 changed = True
     out = set()
     for i, line in enumerate(src, 1):
         code = line.split("//")[0]
-        if any(re.search(r"\b%s\s*\(" % f, code) for f in marked) and "__device__" not in code:
+        if any(re.search(r"\b%s\s*(?:<[^<>()]*>)?\s*\(" % f, code) for f in marked) and \
+                "__device__" not in code:
             out.add(i)
     return out
 

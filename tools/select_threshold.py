@@ -84,7 +84,7 @@ def main():
     if "mcml" in a.what:
         sample = mc_sample(a.mc_warps, a.mc_iters)
         # the PDOM kernel ignores the unroll; SPEC runs U steps per release
-        fams["mcml"] = (r"mcml_pdomILb0ELb0", r"mcml_specILb0ELb0",
+        fams["mcml"] = (r"mcml_pdomILb0ELb0ELb1", r"mcml_specILb0ELb0ELb1",
                         lambda mode, T: mc_warps(sample, a.mc_iters, mode, T,
                                                  a.unroll if mode == oracle.SPEC_LOOP else 1),
                         sample[3] * a.mc_iters)

@@ -100,10 +100,10 @@ CASES = {
     "divloop_spec(T=16)": (r"divloop_specILi125ELb0", lambda: divloop_warps(oracle.SPEC_LOOP, 16)),
     "commoncall_pdom": (r"commoncall_pdomILi250ELb0", lambda: commoncall_warps(oracle.PDOM)),
     "commoncall_spec": (r"commoncall_specILi250ELb0", lambda: commoncall_warps(oracle.SPEC_CALL)),
-    "mcml_pdom_static": (r"mcml_pdomILb0ELb0", lambda: mcml_warps(oracle.PDOM, 0)),
-    "mcml_spec_static(T=32)": (r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 32)),
-    "mcml_spec_static(T=8)": (r"mcml_specILb0ELb0", lambda: mcml_warps(oracle.SPEC_LOOP, 8)),
-    "mcml_spec_static(T=32,U=4)": (r"mcml_specILb0ELb0",
+    "mcml_pdom_static": (r"mcml_pdomILb0ELb0ELb1", lambda: mcml_warps(oracle.PDOM, 0)),
+    "mcml_spec_static(T=32)": (r"mcml_specILb0ELb0ELb1", lambda: mcml_warps(oracle.SPEC_LOOP, 32)),
+    "mcml_spec_static(T=8)": (r"mcml_specILb0ELb0ELb1", lambda: mcml_warps(oracle.SPEC_LOOP, 8)),
+    "mcml_spec_static(T=32,U=4)": (r"mcml_specILb0ELb0ELb1",
                                    lambda: mcml_warps(oracle.SPEC_LOOP, 32, U=4)),
     "rs_pdom": (r"rs_pdomILi8ELi0ELb0", lambda: rsbench_warps(oracle.PDOM, 0)),
     "rs_spec(T=24)": (r"rs_specILi8ELi0ELb0", lambda: rsbench_warps(oracle.SPEC_LOOP, 24)),
