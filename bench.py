@@ -495,8 +495,13 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
     for name, mode, thr in (("pdom", sr.PDOM, 0), (f"spec_t{c.threshold}", sr.SPEC_LOOP,
                                                    c.threshold)):
         t = graph_time(w, c.n_threads, c.iters, mode, thr, reps=5)
-        res[name] = {"value": c.n_threads * c.iters / (t * 1e-3), "unit": "lookups/s", "ms": t}
+        sr.sr_run(w, c.n_threads, c.iters, I.PRIMARY_SEED, mode, thr)
+        nucs = int(ctx.region(w, c.n_threads, sr.T_COUNTERS, torch.int64)[0].item())
+        # FMA roofline: every nuclide body is fma_count FMAs (FFMA2, reading R8)
+        res[name] = {"value": c.n_threads * c.iters / (t * 1e-3), "unit": "lookups/s", "ms": t,
+                     "fma_frac_of_peak": nucs * c.fma_count / (t * 1e-3) / fma_peak}
     res["speedup_vs_pdom"] = res[f"spec_t{c.threshold}"]["value"] / res["pdom"]["value"]
+    res["nuclides"] = nucs
     out["rsbench"] = res
 
     # ... with an expensive task fetch (2048-FMA prolog, Fig. 9's XSBench case):
@@ -530,6 +535,17 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
                      "rays": int(cnt[1]), "node_visits": int(cnt[2]), "tri_tests": int(cnt[3]),
                      "launch": sr.sr_last_launch()}
     res["speedup_vs_pdom"] = res[sname]["value"] / res["pdom"]["value"]
+    # issue roofline (as MC): useful work = the PDOM kernel's thread-instructions per
+    # path (ncu, profiles/simt_efficiency.json), peak = 592 SMSPs x 32 lanes x f
+    simt = load_json(os.path.join(ROOT, "profiles", "simt_efficiency.json")) or {}
+    ti = (simt.get("pt_pdom") or {}).get("thread_inst")
+    if ti:
+        per_path = ti / (c.n_pixels * c.spp)
+        peak = 592 * 32 * f_mhz * 1e6
+        res["issue_roofline"] = {
+            "thread_inst_per_path": per_path,
+            "frac": {k: per_path * res[k]["value"] / peak for k in ("pdom", sname)},
+            "basis": "PDOM thread-inst per path (ncu) x paths/s / (592 x 32 x sm_max_mhz)"}
     out["pathtrace"] = res
     return out
 
