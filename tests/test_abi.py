@@ -169,3 +169,10 @@ def test_sass_is_sm100a_and_uses_the_intended_instructions():
             for l in ff:
                 addend = re.search(r"FFMA2\s+[^;]*,\s*([^,;]+);", l).group(1)
                 assert addend.strip().startswith("UR"), (f, l)
+    # the FAST MC kernels drop the FCHK range checks and slow-path
+    # branches of the path length, the log's s and both Henyey-Greenstein divisions
+    for f in funcs:
+        m = re.search(r"(mcml_(?:pdom|spec)ILb[01]ELb[01]E)Lb1E", f)
+        if m:
+            guarded = next(g for g in funcs if m.group(1) + "Lb0E" in g)
+            assert ops(r"\bFCHK\b", guarded) - ops(r"\bFCHK\b", f) >= 3, f
