@@ -43,14 +43,16 @@ constexpr float kDetEps = 1.0e-12f;
 constexpr uint32_t kMaxStack = 256;
 // CTAs of 128 threads per SM the register budget must allow, per kernel, each
 // at its best measured setting (profiles/pt_tuning_r01.md): both latency-bound
-// kernels want 8 (64 registers; the merged kernel spills 32 bytes and is still
-// faster than at 6 CTAs / 80 registers: 37.3 vs 41.1 ms at T = 12).
+// kernels want as many warps as fit.  With the ray kept once (Path.o/d, not
+// copied into Trav) and the pixel sum accumulated in the output, 9 CTAs
+// (56 registers, 32-40 B spilled) beat 8 (64 registers): SPEC 36.4 -> 35.6 ms,
+// PDOM 67.8 -> 67.0 ms; 10 CTAs (48 registers, 64-80 B spilled) lose (37.5 / 71.2).
 // (An L1 prefetch of the next node / triangle was measured 5 % slower.)
 #ifndef SR_PT_MINB_PDOM
-#define SR_PT_MINB_PDOM 8
+#define SR_PT_MINB_PDOM 9
 #endif
 #ifndef SR_PT_MINB_SPEC
-#define SR_PT_MINB_SPEC 8
+#define SR_PT_MINB_SPEC 9
 #endif
 
 struct V3 {
@@ -178,7 +180,7 @@ __device__ __forceinline__ void tri_test(const PtTri& T, int32_t at, V3 o, V3 d,
 // consecutive banks), so the per-lane traversal state that stays in
 // registers is small and the node fetches have L1 to themselves.
 struct Trav {
-  V3 o, d, inv;
+  V3 inv;           // the ray itself (origin, direction) is the caller's (Path.o, Path.d)
   float tb;
   int32_t ib;       // original index of the closest triangle so far (-1: none)
   uint32_t mb, slot;
@@ -197,9 +199,7 @@ __device__ __forceinline__ int32_t& stk(int32_t i) {
   return pt_stack_smem[(uint32_t)i * blockDim.x + threadIdx.x];
 }
 
-__device__ __forceinline__ void trav_begin(Trav& tr, V3 o, V3 d) {
-  tr.o = o;
-  tr.d = d;
+__device__ __forceinline__ void trav_begin(Trav& tr, V3 d) {
   tr.inv = mk(1.0f / d.x, 1.0f / d.y, 1.0f / d.z);
   tr.tb = INFINITY;
   tr.ib = -1;
@@ -212,22 +212,22 @@ __device__ __forceinline__ void trav_begin(Trav& tr, V3 o, V3 d) {
 }
 
 // returns false when the traversal is finished
-__device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) {
+__device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
   const PtNode N = load_node(a.nodes, tr.node);
   ++st.nodes;
   float tn0, tn1;
-  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, tr.o, tr.inv, tr.tb, tn0);
-  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, tr.o, tr.inv, tr.tb, tn1);
+  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0);
+  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1);
   // leaves: test their triangles now; inner children: descend / push
   if (h0 && N.cnt0 > 0) {
     for (int32_t k = 0; k < N.cnt0; ++k) {
-      tri_test(load_tri(a.tris, N.ref0 + k), N.ref0 + k, tr.o, tr.d, tr.tb, tr.ib, tr.mb, tr.slot);
+      tri_test(load_tri(a.tris, N.ref0 + k), N.ref0 + k, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
       ++st.tests;
     }
   }
   if (h1 && N.cnt1 > 0) {
     for (int32_t k = 0; k < N.cnt1; ++k) {
-      tri_test(load_tri(a.tris, N.ref1 + k), N.ref1 + k, tr.o, tr.d, tr.tb, tr.ib, tr.mb, tr.slot);
+      tri_test(load_tri(a.tris, N.ref1 + k), N.ref1 + k, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
       ++st.tests;
     }
   }
@@ -256,12 +256,12 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, Stats& st) 
 // the next node exactly as trav_step (node = -1 when the stack is empty).
 // trav_leaf tests ONE queued triangle.  Returns: a leaf triangle is pending
 // (na > 0), else a node is pending (node >= 0), else the traversal is done.
-__device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, Stats& st) {
+__device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats& st) {
   const PtNode N = load_node(a.nodes, tr.node);
   ++st.nodes;
   float tn0, tn1;
-  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, tr.o, tr.inv, tr.tb, tn0);
-  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, tr.o, tr.inv, tr.tb, tn1);
+  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0);
+  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1);
   const bool l0 = h0 && N.cnt0 > 0, l1 = h1 && N.cnt1 > 0;
   tr.la = l0 ? N.ref0 : N.ref1;
   tr.na = l0 ? (uint32_t)N.cnt0 : (l1 ? (uint32_t)N.cnt1 : 0u);
@@ -282,8 +282,8 @@ __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, Stats& st) 
   tr.node = next;
 }
 
-__device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, Stats& st) {
-  tri_test(load_tri(a.tris, tr.la), tr.la, tr.o, tr.d, tr.tb, tr.ib, tr.mb, tr.slot);
+__device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
+  tri_test(load_tri(a.tris, tr.la), tr.la, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
   ++st.tests;
   ++tr.la;
   if (--tr.na == 0u) {
@@ -294,14 +294,14 @@ __device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, Stats& st) 
 }
 
 __device__ __forceinline__ int64_t closest_hit(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
-  trav_begin(tr, o, d);
-  while (trav_step(a, tr, st)) {
+  trav_begin(tr, d);
+  while (trav_step(a, tr, o, d, st)) {
   }
   return (int64_t)tr.ib;
 }
 
 struct Path {
-  V3 o, d, thr, rad, sum;
+  V3 o, d, thr, rad;   // the pixel sum lives in a.rgb (this lane's pixel only)
   uint32_t pix, s, b;
   bool alive;
 };
@@ -396,7 +396,12 @@ __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
   p.b = p.b + 1u;
   if (!end && p.b >= a.max_depth) end = true;
   if (end) {
-    p.sum = add(p.sum, p.rad);   // Epilog: pixel += radiance (sample order)
+    // Epilog: pixel += radiance, in sample order, in the output itself (a lane owns
+    // its pixel; one read-modify-write per path keeps three registers free)
+    float* px = a.rgb + 3 * (uint64_t)p.pix;
+    px[0] = px[0] + p.rad.x;
+    px[1] = px[1] + p.rad.y;
+    px[2] = px[2] + p.rad.z;
     p.alive = false;
   }
 }
@@ -406,11 +411,6 @@ __device__ __forceinline__ void finish(const PtArgs& a, const Path& p, bool vali
                                        uint32_t rel, uint32_t rel_lanes, uint32_t adv,
                                        uint32_t adv_lanes, uint32_t lrel = 0,
                                        uint32_t lrel_lanes = 0) {
-  if (valid) {
-    a.rgb[3 * (uint64_t)p.pix + 0] = p.sum.x;
-    a.rgb[3 * (uint64_t)p.pix + 1] = p.sum.y;
-    a.rgb[3 * (uint64_t)p.pix + 2] = p.sum.z;
-  }
   unsigned long long v[4] = {paths, st.rays, st.nodes, st.tests};
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
@@ -441,7 +441,10 @@ __global__ void __launch_bounds__(128, SR_PT_MINB_PDOM) pt_pdom(const PtArgs a) 
   const bool valid = g < a.n;
   Path p;
   p.pix = (uint32_t)(valid ? g : 0);
-  p.sum = mk(0.0f, 0.0f, 0.0f);
+  if (valid) {
+    float* px = a.rgb + 3 * (uint64_t)p.pix;
+    px[0] = 0.0f; px[1] = 0.0f; px[2] = 0.0f;
+  }
   p.alive = false;
   Trav tr;
   Stats st{0, 0, 0};
@@ -481,7 +484,10 @@ __global__ void __launch_bounds__(128, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) 
   const bool valid = g < a.n;
   Path p;
   p.pix = (uint32_t)(valid ? g : 0);
-  p.sum = mk(0.0f, 0.0f, 0.0f);
+  if (valid) {
+    float* px = a.rgb + 3 * (uint64_t)p.pix;
+    px[0] = 0.0f; px[1] = 0.0f; px[2] = 0.0f;
+  }
   p.alive = false;
   p.s = 0;
   Trav tr;
@@ -508,11 +514,11 @@ __global__ void __launch_bounds__(128, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) 
           __syncwarp(G);
           if (leaf) {
             if constexpr (SCHED) { ++lrel; lrel_lanes += __popc(G); }
-            for (uint32_t k = 0; k < a.unroll && tr.na > 0u; ++k) trav_leaf(a, tr, st);
+            for (uint32_t k = 0; k < a.unroll && tr.na > 0u; ++k) trav_leaf(a, tr, p.o, p.d, st);
           } else {
             if constexpr (SCHED) { ++rel; rel_lanes += __popc(G); }
             for (uint32_t k = 0; k < a.unroll && tr.na == 0u && tr.node >= 0; ++k)
-              trav_node(a, tr, st);
+              trav_node(a, tr, p.o, st);
           }
           trav = tr.na > 0u || tr.node >= 0;
         }
@@ -527,7 +533,7 @@ __global__ void __launch_bounds__(128, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) 
           ++paths;
         }
         if (p.alive) {
-          trav_begin(tr, p.o, p.d);
+          trav_begin(tr, p.d);
           ++st.rays;
           trav = true;
         }
@@ -544,7 +550,7 @@ __global__ void __launch_bounds__(128, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) 
       if ((P >> lane_id()) & 1u) {
         __syncwarp(P);
         if constexpr (NODE) {
-          for (uint32_t k = 0; k < a.unroll && trav; ++k) trav = trav_step(a, tr, st);
+          for (uint32_t k = 0; k < a.unroll && trav; ++k) trav = trav_step(a, tr, p.o, p.d, st);
         }
         else bounce(a, p, tr, st);
       }
@@ -558,7 +564,7 @@ __global__ void __launch_bounds__(128, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) 
           ++paths;
         }
         if (NODE && p.alive) {                        // start the next ray
-          trav_begin(tr, p.o, p.d);
+          trav_begin(tr, p.d);
           ++st.rays;
           trav = true;
         }

@@ -21,6 +21,8 @@ VARIANTS = {
     "libsr_pts7.so": ["SR_PT_MINB_SPEC=7"],
     "libsr_pts8.so": ["SR_PT_MINB_SPEC=8"],
     "libsr_ptp6.so": ["SR_PT_MINB_PDOM=6"],
+    "libsr_pt9.so": ["SR_PT_MINB_SPEC=9", "SR_PT_MINB_PDOM=9"],
+    "libsr_pt10.so": ["SR_PT_MINB_SPEC=10", "SR_PT_MINB_PDOM=10"],
 }
 if __name__ == "__main__":
     names = sys.argv[1:] or list(VARIANTS)
