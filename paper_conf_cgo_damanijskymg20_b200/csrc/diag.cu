@@ -48,6 +48,15 @@ __global__ void math_eval_p_kernel(int fn, float p, const float* __restrict__ x,
         r = sqrt_dom(1.0f - c * c);
         break;
       }
+      case SR_FNP_DIV2_XP: {   // pairs (x[2j], x[2j+1]) / p through div2_dom
+        if (i & 1u) continue;
+        const uint64_t q = div2_dom(pack2(v, i + 1 < n ? x[i + 1] : 1.0f), p);
+        float q0, q1;
+        unpack2(q, q0, q1);
+        out[i] = q0;
+        if (i + 1 < n) out[i + 1] = q1;
+        continue;
+      }
       default: r = 0.0f; break;
     }
     out[i] = r;

@@ -169,7 +169,7 @@ int sr_math_eval(int fn, const float* x_dev, float* out_dev, uint64_t n) {
 int sr_math_eval_p(int fn, float p, const float* x_dev, float* out_dev, uint64_t n) {
   std::lock_guard<std::mutex> lk(g_mu);
   g_err.clear();
-  if (fn < SR_FNP_DIV_XP || fn > SR_FNP_HG_SINT) return fail(SR_E_INVALID, "unknown fn");
+  if (fn < SR_FNP_DIV_XP || fn > SR_FNP_DIV2_XP) return fail(SR_E_INVALID, "unknown fn");
   if (n && (!x_dev || !out_dev)) return fail(SR_E_INVALID, "NULL array");
   if (!g_ctx.live) return fail(SR_E_STATE, "sr_math_eval_p before sr_init");
   if (!n) return SR_OK;

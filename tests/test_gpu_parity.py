@@ -113,6 +113,16 @@ def test_div_dom_log_uniform_operands(ctx, p):
         assert_bits(got, pf / x[3:], x[3:])
 
 
+@pytest.mark.parametrize("p", [1.41e-3, 0.37, 1.0, 0.999999])
+def test_div2_dom_rotation_quotients(ctx, p):
+    """the rotation's paired quotients t / sqrt(1 - uz^2): |t| in [2^-100, 2], divisor in
+    [1.41e-3, 1] -- 2^22 log-uniform numerators of both signs, lane by lane == IEEE"""
+    rng = np.random.default_rng(11)
+    n = 1 << 22
+    x = (np.exp2(rng.uniform(-100, 1, n)) * rng.choice([-1.0, 1.0], n)).astype(F32)
+    assert_bits(eval_p(ctx, sr.FNP_DIV2_XP, p, x), x / F32(p), x)
+
+
 def test_sqrt_dom_matches_ieee(ctx):
     """every binary32 in [2^-25, 1) (the 1 - c^2 arguments), +0, and 2^22 log-uniform
     values over [2^-101, 2^127]"""

@@ -90,6 +90,8 @@ def predicted_regions(label, costs_all):
             name, full = key.split(":")[0], key.endswith(":full")
             if name in ("ENTRY", "UNMAPPED"):
                 x, l = 1, nv
+            elif name.startswith("COLD"):
+                x, l = 0, 0
             else:
                 x, ln = sim[name]
                 l = x * nv if full else ln

@@ -34,6 +34,10 @@ def accumulate(costs, sim, n_valid, acc):
         name, full = key.split(":")[0], key.endswith(":full")
         if name in ("ENTRY", "UNMAPPED"):
             x, l = 1, n_valid
+        elif name.startswith("COLD"):
+            # the guarded slow branch of a domain check that the workloads never
+            # take: no executions
+            x, l = 0, 0
         else:
             x, ln = sim[name]
             l = x * n_valid if full else ln
