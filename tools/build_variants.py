@@ -21,6 +21,9 @@ VARIANTS = {
     "libsr_pts7.so": ["SR_PT_MINB_SPEC=7"],
     "libsr_pts8.so": ["SR_PT_MINB_SPEC=8"],
     "libsr_ptp6.so": ["SR_PT_MINB_PDOM=6"],
+    "libsr_ch16.so": ["SR_MC_CHUNK=16"],
+    "libsr_ch32.so": ["SR_MC_CHUNK=32"],
+    "libsr_ch128.so": ["SR_MC_CHUNK=128"],
     "libsr_pt9.so": ["SR_PT_MINB_SPEC=9", "SR_PT_MINB_PDOM=9"],
     "libsr_pt10.so": ["SR_PT_MINB_SPEC=10", "SR_PT_MINB_PDOM=10"],
 }
