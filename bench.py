@@ -490,7 +490,7 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
 
     # NEXT-1: RSBench-shaped nested trip-count loop (Fig. 3), PDOM vs Loop Merge
     c = I.NEXT1
-    w = sr.rsbench_workload(c.fma_count)
+    w = sr.rsbench_workload(c.fma_count, unroll=c.merge_unroll)
     res = {}
     for name, mode, thr in (("pdom", sr.PDOM, 0), (f"spec_t{c.threshold}", sr.SPEC_LOOP,
                                                    c.threshold)):
@@ -507,7 +507,7 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
     # ... with an expensive task fetch (2048-FMA prolog, Fig. 9's XSBench case):
     # refilling idle lanes costs more, the best threshold drops (T = 32 shown too)
     c = I.NEXT1_FETCH
-    w = sr.rsbench_workload(c.fma_count, prolog_fma=c.prolog_fma)
+    w = sr.rsbench_workload(c.fma_count, prolog_fma=c.prolog_fma, unroll=c.merge_unroll)
     res = {"prolog_fma": c.prolog_fma}
     for name, mode, thr in (("pdom", sr.PDOM, 0), (f"spec_t{c.threshold}", sr.SPEC_LOOP,
                                                    c.threshold), ("spec_t32", sr.SPEC_LOOP, 32)):

@@ -122,6 +122,9 @@ typedef struct {
   uint32_t prolog_fma; /* FMAs of the lookup prolog (an expensive task fetch,
                           E = Expensive(E, prolog_fma)); multiple of 8, <= 65536;
                           0 = none (configs: 0; the Fig. 9 XSBench-like sweep: 2048) */
+  uint32_t merge_unroll; /* SR_SPEC_LOOP: inner-loop iterations per release round,
+                          the partial unroll of P:1467-1474 (0 = 1). Results are
+                          identical for every value.                             */
 } sr_rsbench_params;   /* materials / nuclide counts: DESIGN.md reading R8       */
 
 typedef struct {

@@ -259,11 +259,15 @@ def ws_commoncall(arm, mode, W=32):
     return o.as_dict(CC)
 
 
-def ws_loopmerge(nsteps, mode, T, W=32, events=None):
-    """nsteps: [n_valid, K] uint32; events: optional list-of-lists of uint16 arrays."""
+def ws_loopmerge(nsteps, mode, T, W=32, events=None, U=1):
+    """nsteps: [n_valid, K] uint32; events: optional list-of-lists of uint16 arrays;
+    U = inner iterations per release (events=None only)."""
     nsteps = np.ascontiguousarray(nsteps, np.uint32)
     n_valid, K = nsteps.shape
     o = WsCounts()
+    if U != 1:
+        assert events is None
+        return ws_loopmerge_raw(nsteps, None, None, mode, T, W, U)
     if events is not None:
         flat = [events[l][k] for l in range(n_valid) for k in range(K)]
         off = np.zeros(len(flat), np.uint64)
@@ -280,7 +284,8 @@ def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32, U=1):
     """nsteps [n_valid, K]; ev_off [n_valid*K] offsets into the flat event buffer;
     U = steps per release (partial unroll of the merged loop)."""
     nsteps = np.ascontiguousarray(nsteps, np.uint32)
-    ev_off = np.ascontiguousarray(ev_off, np.uint64)
+    if ev_off is not None:
+        ev_off = np.ascontiguousarray(ev_off, np.uint64)
     n_valid, K = nsteps.shape
     o = WsCounts()
     L = lib()
@@ -288,15 +293,18 @@ def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32, U=1):
                                         C.POINTER(C.c_uint64), C.c_uint32, C.c_uint32,
                                         C.c_uint32, C.c_int, C.c_uint32, C.c_uint32,
                                         C.POINTER(WsCounts)]
-    L.ws_loopmerge_unrolled(_p(nsteps, C.c_uint32), _p(ev_flat, C.c_uint16),
-                            _p(ev_off, C.c_uint64), W, n_valid, K, mode, T, U, C.byref(o))
+    L.ws_loopmerge_unrolled(_p(nsteps, C.c_uint32),
+                            None if ev_flat is None else _p(ev_flat, C.c_uint16),
+                            None if ev_off is None else _p(ev_off, C.c_uint64),
+                            W, n_valid, K, mode, T, U, C.byref(o))
     return o.as_dict(LM)
 
 
 def ws_loopmerge_defer_raw(nsteps, ev_flat, ev_off, T, Tb, W=32):
     """Loop Merge + nested Iteration Delay of the boundary sub-step."""
     nsteps = np.ascontiguousarray(nsteps, np.uint32)
-    ev_off = np.ascontiguousarray(ev_off, np.uint64)
+    if ev_off is not None:
+        ev_off = np.ascontiguousarray(ev_off, np.uint64)
     n_valid, K = nsteps.shape
     o = WsCounts()
     L = lib()

@@ -34,6 +34,7 @@ struct RsArgs {
   uint32_t thr[kMats];   // cumulative selection thresholds (host-computed)
   uint32_t iters, rounds, T;
   uint32_t prolog_rounds;  // expensive prolog (task fetch): 0 = none
+  uint32_t unroll;         // inner iterations per release (partial unroll)
   uint2* out;            // {acc bits, nuclides}
   unsigned long long* counters;
   uint32_t* sched;
@@ -131,12 +132,16 @@ __global__ void __launch_bounds__(256) rs_spec(const RsArgs a) {
       if constexpr (SCHED) { ++rel; rel_lanes += __popc(P); }  // @sr-region RELEASE:full
       if (busy) {
         __syncwarp(P);  // @sr-region STEP
-        xs = xs + body<ROUNDS>(E, m, i, a.rounds);
-        i = i + 1u;
-        if (i == N) {                      // inner loop done: Epilog
-          acc = acc + xs;
-          nucs += N;
-          busy = false;
+        // up to `unroll` inner iterations per release; a lane whose lookup ends
+        // inside the release idles for the rest of it
+        for (uint32_t r = 0; r < a.unroll && busy; ++r) {
+          xs = xs + body<ROUNDS>(E, m, i, a.rounds);
+          i = i + 1u;
+          if (i == N) {                    // inner loop done: Epilog
+            acc = acc + xs;
+            nucs += N;
+            busy = false;
+          }
         }
       }
     } else {
@@ -196,6 +201,7 @@ cudaError_t launch_rsbench(const LaunchCtx& c, const sr_workload& w, uint64_t n,
   a.iters = iters;
   a.rounds = w.rsbench.fma_count / 8u;
   a.prolog_rounds = w.rsbench.prolog_fma / 8u;
+  a.unroll = w.rsbench.merge_unroll ? w.rsbench.merge_unroll : 1u;
   a.T = T;
   a.out = reinterpret_cast<uint2*>(c.ws + c.lay.off[SR_T_PERTHREAD]);
   a.counters = reinterpret_cast<unsigned long long*>(c.ws + c.lay.off[SR_T_COUNTERS]);

@@ -42,6 +42,7 @@ class RSBench:
     fma_count: int = 64         # FMAs of the per-nuclide body
     threshold: int = 24         # best of the sweep (profiles/threshold_sweep_*.md)
     prolog_fma: int = 0         # FMAs of the lookup prolog (expensive task fetch)
+    merge_unroll: int = 12      # inner iterations per release, tuned on B200
 
 
 NEXT1 = RSBench()

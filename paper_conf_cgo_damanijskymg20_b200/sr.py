@@ -65,7 +65,8 @@ class PathtraceParams(C.Structure):
 
 
 class RsbenchParams(C.Structure):
-    _fields_ = [("fma_count", C.c_uint32), ("prolog_fma", C.c_uint32)]
+    _fields_ = [("fma_count", C.c_uint32), ("prolog_fma", C.c_uint32),
+                ("merge_unroll", C.c_uint32)]
 
 
 class Workload(C.Structure):
@@ -211,9 +212,10 @@ def divloop_workload(p_u32=1 << 29, fma_count=1000, task_offset=0, flags=0, bloc
     return w
 
 
-def rsbench_workload(fma_count=64, task_offset=0, flags=0, block=0, prolog_fma=0) -> Workload:
+def rsbench_workload(fma_count=64, task_offset=0, flags=0, block=0, prolog_fma=0,
+                     unroll=0) -> Workload:
     w = Workload(kind=WL_RSBENCH, flags=flags, task_offset=task_offset, block_threads=block)
-    w.rsbench = RsbenchParams(fma_count, prolog_fma)
+    w.rsbench = RsbenchParams(fma_count, prolog_fma, unroll)
     return w
 
 

@@ -44,6 +44,31 @@ def test_rsbench_bit_exact_small(ctx, seed, mode, T):
     assert cnt[0] == nuc_o.sum()
 
 
+@pytest.mark.parametrize("T,U", [(24, 2), (32, 3), (4, 4)])
+def test_rsbench_unrolled_merge_bit_exact(ctx, T, U):
+    """up to U inner iterations per release: same bits"""
+    n, iters = 700, 6
+    acc_o, nuc_o = oracle.rsbench(3, n, iters, 9)
+    acc, nuc, cnt = run(ctx, sr.rsbench_workload(block=64, task_offset=3, unroll=U), n, iters,
+                        9, sr.SPEC_LOOP, T)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(nuc, nuc_o)
+
+
+@pytest.mark.parametrize("T,U", [(24, 2), (32, 4)])
+def test_rsbench_unrolled_schedule_matches_simulator(ctx, T, U):
+    n, iters = 256, 8
+    w = sr.rsbench_workload(flags=sr.F_SCHED, block=64, unroll=U)
+    run(ctx, w, n, iters, 5, sr.SPEC_LOOP, T)
+    sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    _, _, trips = oracle.rsbench(0, n, iters, 5, fma_count=0, trips=True)
+    for wi in range(n // 32):
+        s = oracle.ws_loopmerge(trips[32 * wi:32 * wi + 32], oracle.SPEC_LOOP, T, U=U)
+        g = sched[wi]
+        assert g[0] == s["rounds"] and (g[1], g[2]) == s["RELEASE"], wi
+        assert (g[3], g[4]) == s["LAUNCH"], wi
+
+
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 4), (sr.SPEC_LOOP, 32)])
 def test_rsbench_schedule_matches_simulator(ctx, mode, T):
     n, iters = 256, 8

@@ -53,7 +53,7 @@ if "mcml" in a.what:
                   0 if md == "pdom" else a.threshold)
 if "rsbench" in a.what:
     c = I.NEXT1
-    w = sr.rsbench_workload(c.fma_count)
+    w = sr.rsbench_workload(c.fma_count, unroll=c.merge_unroll)
     ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
     for md in modes:
         sr.sr_run(w, c.n_threads, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,

@@ -91,12 +91,13 @@ def mcml_warps(mode, T, n_threads=MC_VALIDATION["n_threads"], iters=MC_VALIDATIO
         yield oracle.ws_loopmerge_raw(ns[ids], ev, off[ids].ravel(), mode, T, U=U), len(lanes)
 
 
-def rsbench_warps(mode, T):
+def rsbench_warps(mode, T, U=None):
     c = I.NEXT1
+    U = c.merge_unroll if U is None else U
     _, _, trips = oracle.rsbench(0, c.n_threads, c.iters, I.PRIMARY_SEED, fma_count=0, trips=True)
     for w in range(0, c.n_threads, 32):
         tr = trips[w:w + 32]
-        yield oracle.ws_loopmerge(tr, mode, T), len(tr)
+        yield oracle.ws_loopmerge(tr, mode, T, U=U if mode == oracle.SPEC_LOOP else 1), len(tr)
 
 
 CASES = {

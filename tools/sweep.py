@@ -24,7 +24,7 @@ ap.add_argument("--blocks", default="0")
 ap.add_argument("--photons", type=int, default=I.C3.n_photons)
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--flags", type=int, default=0, help="extra sr_workload.flags (e.g. 4 = F_COARSE)")
-ap.add_argument("--unroll", type=int, default=0, help="PT node-merge partial unroll")
+ap.add_argument("--unroll", type=int, default=0, help="merge partial unroll (MC steps, PT node visits, RSBench inner iterations per release)")
 ap.add_argument("--defer", type=int, default=0, help="MCML boundary defer threshold T_b")
 ap.add_argument("--static", action="store_true", help="MCML static photon assignment (F_STATIC)")
 ap.add_argument("--iters", type=int, default=0, help="MCML photons per lane (default configs[2])")
@@ -106,7 +106,7 @@ if "rsbench" in a.what:
     c = I.NEXT1
     res = []
     for b in blocks:
-        w = sr.rsbench_workload(c.fma_count, block=b, prolog_fma=a.prolog)
+        w = sr.rsbench_workload(c.fma_count, block=b, prolog_fma=a.prolog, unroll=a.unroll)
         ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
             t = timed(lambda: sr.sr_run(w, c.n_threads, c.iters, seed, mode, T), a.reps)
