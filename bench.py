@@ -460,21 +460,22 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
         return statistics.median(ms) / reps
 
     c = I.C1
-    w = sr.divloop_workload(c.p_u32, c.fma_count)
+    w = sr.divloop_workload(c.p_u32, c.fma_count, advance=c.advance_unroll)
     n_units = c.n_threads * c.iters
     exp_calls = None
     res = {}
-    # T = 16 is the config's threshold; T = 12 the best of the sweep
-    # (profiles/threshold_sweep_r01h.md); T = 32 = wait for every lane (Fig. 1(b))
+    # T = 16 is the config's threshold; T = 8 the best of the sweep with run-ahead lanes
+    # taking up to 8 iterations per round (tools/exp_dl_adv.sh); T = 32 = wait for every
+    # lane (Fig. 1(b))
     for name, mode, thr in (("pdom", sr.PDOM, 0), ("spec_t16", sr.SPEC_LOOP, 16),
-                            ("spec_t12", sr.SPEC_LOOP, 12), ("spec_t32", sr.SPEC_LOOP, 32)):
+                            ("spec_t8", sr.SPEC_LOOP, 8), ("spec_t32", sr.SPEC_LOOP, 32)):
         t = graph_time(w, c.n_threads, c.iters, mode, thr)
         sr.sr_run(w, c.n_threads, c.iters, I.PRIMARY_SEED, mode, thr)
         exp_calls = int(ctx.region(w, c.n_threads, sr.T_COUNTERS, torch.int64)[0].item())
         res[name] = {"value": n_units / (t * 1e-3), "unit": "thread-iterations/s", "ms": t,
                      "fma_frac_of_peak": exp_calls * c.fma_count / (t * 1e-3) / fma_peak}
     res["speedup_t16_vs_pdom"] = res["spec_t16"]["value"] / res["pdom"]["value"]
-    res["speedup_t12_vs_pdom"] = res["spec_t12"]["value"] / res["pdom"]["value"]
+    res["speedup_t8_vs_pdom"] = res["spec_t8"]["value"] / res["pdom"]["value"]
     res["expensive_calls"] = exp_calls
     out["divloop"] = res
 

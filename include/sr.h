@@ -82,6 +82,9 @@ typedef struct { float n, mua, mus, g, d; } sr_layer;  /* -, 1/cm, 1/cm, -, cm *
 typedef struct {
   uint32_t p_u32;      /* P(condition) = p_u32 / 2^32 (1/8: 2^29)               */
   uint32_t fma_count;  /* FMAs in Expensive(); multiple of 8 (1000)             */
+  uint32_t advance_unroll; /* SR_SPEC_LOOP: iterations a run-ahead lane may take in
+                          one advance round before it parks (0 = 1, reading Q5).
+                          Results are identical for every value.               */
 } sr_divloop_params;
 
 typedef struct {

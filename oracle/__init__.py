@@ -98,6 +98,8 @@ def lib():
         L.or_mcml_rsp.argtypes = [C.POINTER(MCParams)]; L.or_mcml_rsp.restype = C.c_float
         L.ws_divloop.argtypes = [u8p, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int, C.c_uint32,
                                  C.POINTER(WsCounts)]
+        L.ws_divloop_adv.argtypes = [u8p, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int,
+                                     C.c_uint32, C.c_uint32, C.POINTER(WsCounts)]
         L.ws_commoncall.argtypes = [u8p, C.c_uint32, C.c_uint32, C.c_int, C.POINTER(WsCounts)]
         L.ws_loopmerge.argtypes = [u32p, C.POINTER(C.c_uint16), u64p, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int,
                                    C.c_uint32, C.POINTER(WsCounts)]
@@ -244,11 +246,13 @@ def mcml_rsp(p: MCParams) -> float:
 
 
 # ---------------------------------------------------------------- simulator
-def ws_divloop(want, mode, T, W=32, n_valid=None):
+def ws_divloop(want, mode, T, W=32, n_valid=None, V=1):
+    """V = iterations a run-ahead lane may take per advance round (1: reading Q5)."""
     want = np.ascontiguousarray(want, np.uint8)
     n_valid = want.shape[0] if n_valid is None else n_valid
     o = WsCounts()
-    lib().ws_divloop(_p(want, C.c_uint8), W, n_valid, want.shape[1], mode, T, C.byref(o))
+    lib().ws_divloop_adv(_p(want, C.c_uint8), W, n_valid, want.shape[1], mode, T, V,
+                         C.byref(o))
     return o.as_dict(DL)
 
 

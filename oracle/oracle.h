@@ -163,6 +163,8 @@ typedef struct {
 } ws_counts;
 /* One warp of W<=32 lanes, lane l valid iff l < n_valid.
  * want[l*L + i] = lane l takes the branch in iteration i. */
+void ws_divloop_adv(const uint8_t* want, uint32_t W, uint32_t n_valid, uint32_t L, int mode,
+                    uint32_t T, uint32_t V, ws_counts* o);
 void ws_divloop(const uint8_t* want, uint32_t W, uint32_t n_valid, uint32_t L,
                 int mode, uint32_t T, ws_counts* out);
 /* arm[l] = 1 if lane l takes the then-arm (Fig. 2(c) line 8) */

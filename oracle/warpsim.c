@@ -43,7 +43,15 @@ static void hit(ws_counts* o, int r, uint32_t mask) {
 /* Iteration Delay: Fig. 2(a) / Listing 1.                              */
 void ws_divloop(const uint8_t* want, uint32_t W, uint32_t n_valid, uint32_t L, int mode,
                 uint32_t T, ws_counts* o) {
+  ws_divloop_adv(want, W, n_valid, L, mode, T, 1, o);
+}
+
+/* V > 1: in an advance round a run-ahead lane takes up to V iterations, stopping
+ * at the first one that wants Expensive (it parks there). */
+void ws_divloop_adv(const uint8_t* want, uint32_t W, uint32_t n_valid, uint32_t L, int mode,
+                    uint32_t T, uint32_t V, ws_counts* o) {
   memset(o, 0, sizeof *o);
+  if (V == 0) V = 1;
   if (n_valid > W) n_valid = W;
   uint32_t valid = n_valid >= 32 ? 0xffffffffu : ((1u << n_valid) - 1u);
   hit(o, WS_DL_ENTRY, valid);
@@ -77,14 +85,17 @@ void ws_divloop(const uint8_t* want, uint32_t W, uint32_t n_valid, uint32_t L, i
       parked = 0;
     } else {
       hit(o, WS_DL_ADVANCE, R);
-      hit(o, WS_DL_PROLOG, R);
-      uint32_t E = 0;
-      for (uint32_t l = 0; l < n_valid; ++l) {
-        if (!(R >> l & 1u)) continue;
-        if (want[l * L + it[l]]) parked |= 1u << l;   /* Join + Wait at L1 */
-        else { E |= 1u << l; it[l] += 1; }             /* run ahead */
+      uint32_t S = R;   /* lanes still running ahead in this round */
+      for (uint32_t v = 0; v < V && S; ++v) {
+        hit(o, WS_DL_PROLOG, S);
+        uint32_t E = 0;
+        for (uint32_t l = 0; l < n_valid; ++l) {
+          if (!(S >> l & 1u)) continue;
+          if (want[l * L + it[l]]) { parked |= 1u << l; S &= ~(1u << l); } /* Join + Wait */
+          else { E |= 1u << l; it[l] += 1; if (it[l] >= L) S &= ~(1u << l); } /* run ahead */
+        }
+        hit(o, WS_DL_EPILOG, E);
       }
-      hit(o, WS_DL_EPILOG, E);
     }
   }
 }

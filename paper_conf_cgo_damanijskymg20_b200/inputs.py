@@ -22,6 +22,7 @@ class DivLoop:
     p_u32: int = 1 << 29        # P(branch) = 1/8 exactly
     fma_count: int = 1000       # Expensive() = 1000 FMAs
     threshold: int = 16
+    advance_unroll: int = 8     # iterations a run-ahead lane may take per round, tuned on B200
 
 
 @dataclass(frozen=True)

@@ -212,6 +212,31 @@ def test_divloop_edge_cases(ctx, kw, n, iters, off, mode, T):
     assert np.array_equal(cnt, cnt_o)
 
 
+
+@pytest.mark.parametrize("T,V", [(16, 2), (16, 8), (32, 4), (4, 64)])
+def test_divloop_advance_unroll_bit_exact(ctx, T, V):
+    """run-ahead lanes taking up to V iterations per advance round: same bits"""
+    n, iters = 1000, 64
+    acc_o, cnt_o = oracle.divloop(0, n, iters, 7)
+    acc, cnt, _ = run_divloop(ctx, sr.divloop_workload(block=64, advance=V), n, iters, 7,
+                              sr.SPEC_LOOP, T)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(cnt, cnt_o)
+
+
+@pytest.mark.parametrize("T,V", [(16, 2), (16, 4), (32, 8)])
+def test_divloop_advance_unroll_schedule_matches_simulator(ctx, T, V):
+    n, iters = 2000, 64
+    w = sr.divloop_workload(flags=sr.F_SCHED, block=64, advance=V)
+    run_divloop(ctx, w, n, iters, I.PRIMARY_SEED, sr.SPEC_LOOP, T)
+    sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    want = oracle.divloop_wants(0, n, iters, I.PRIMARY_SEED)
+    for wi in range((n + 31) // 32):
+        s = oracle.ws_divloop(want[32 * wi:32 * wi + 32], oracle.SPEC_LOOP, T, V=V)
+        g = sched[wi]
+        assert (g[1], g[2]) == s["EXPENSIVE"], wi
+        assert g[0] == s["rounds"] and (g[3], g[4]) == s["ADVANCE"], wi
+
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 16),
                                     (sr.SPEC_LOOP, 32)])
 def test_divloop_schedule_matches_simulator(ctx, mode, T):

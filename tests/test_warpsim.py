@@ -167,3 +167,20 @@ def test_loopmerge_defer_groups_boundaries():
     defer = oracle.ws_loopmerge_defer_raw(ns[ids], ev, off[ids].ravel(), 32, 8)
     eff = lambda x: x[1] / max(1, 32 * x[0])
     assert eff(defer["B_REL"]) > 4 * eff(plain["STEP_BOUNDARY"])
+
+
+def test_divloop_advance_unroll_invariants():
+    """V iterations per advance round: every lane-iteration's prolog still
+    runs exactly once, every wanting iteration's Expensive exactly once; at T = 32 the
+    releases (all lanes parked at their next wanting iteration) do not depend on V."""
+    rng = np.random.default_rng(5)
+    want = (rng.random((32, 64)) < 0.125).astype(np.uint8)
+    base = oracle.ws_divloop(want, oracle.SPEC_LOOP, 32)
+    for V in (2, 3, 8, 64):
+        for T in (1, 8, 16, 32):
+            s = oracle.ws_divloop(want, oracle.SPEC_LOOP, T, V=V)
+            assert s["PROLOG"][1] == 32 * 64 - int(want.sum()) + int(want.sum())
+            assert s["EXPENSIVE"][1] == int(want.sum())
+            if T == 32:
+                assert s["EXPENSIVE"] == base["EXPENSIVE"]
+            assert s["rounds"] <= oracle.ws_divloop(want, oracle.SPEC_LOOP, T)["rounds"]

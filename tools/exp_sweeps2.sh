@@ -8,7 +8,7 @@ mkdir -p $O
 S="python tools/sweep.py --reps 3"
 TS=1,2,4,8,12,16,20,24,32
 timeout 900 $S --what mcml --thresholds $TS --unroll 4 > $O/sweep_mc_$TAG.json 2>/dev/null
-timeout 900 $S --what divloop --thresholds $TS > $O/sweep_dl_$TAG.json 2>/dev/null
+timeout 900 $S --what divloop --thresholds $TS --unroll 8 > $O/sweep_dl_$TAG.json 2>/dev/null
 timeout 900 $S --what rsbench --thresholds $TS --unroll 12 > $O/sweep_rs_$TAG.json 2>/dev/null
 timeout 900 $S --what rsbench --thresholds $TS --prolog 2048 --unroll 12 > $O/sweep_rsfetch_$TAG.json 2>/dev/null
 timeout 1200 $S --what pathtrace --thresholds $TS --unroll 8 > $O/sweep_pt_$TAG.json 2>/dev/null

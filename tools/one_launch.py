@@ -30,7 +30,7 @@ ctx = sr.Context.create(0, 1 << 20)
 seed = I.PRIMARY_SEED
 if "divloop" in a.what:
     c = I.C1
-    w = sr.divloop_workload(c.p_u32, c.fma_count)
+    w = sr.divloop_workload(c.p_u32, c.fma_count, advance=c.advance_unroll)
     ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
     for md in modes:
         sr.sr_run(w, c.n_threads, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,

@@ -340,6 +340,31 @@ def kernel_costs(kernel_regex=".*"):
             m = re.match(r"(?:@\S+\s+)?BSYNC(?:\.\w+)?\s+(B\d+)", x["text"])
             if m and m.group(1) in open_bssy:
                 final[i] = open_bssy[m.group(1)]
+        # loop nesting: a region whose code sits mostly in an inner loop (the merged
+        # loop's partial unroll, the run-ahead loop, PDOM's inner do-while) may have
+        # instructions the compiler hoisted into the enclosing loop; those run once
+        # per entry of the inner loop -- per release / advance round / launch -- with
+        # that step's lanes, so they are costed to the entering region
+        regions_here = {f[0] for f in final if f is not None}
+        enter = {"STEP": "RELEASE" if "RELEASE" in regions_here else "LAUNCH",
+                 "PROLOG": "ADVANCE"}
+        for rname, ename in enter.items():
+            if ename not in regions_here and ename != "LAUNCH":
+                continue
+            idx = [i for i in range(len(body)) if final[i] is not None and final[i][0] == rname
+                   and i not in cold]
+            if not idx:
+                continue
+            inner = [(a_, b_) for a_, b_ in loops
+                     if sum(a_ <= i <= b_ for i in idx) * 2 > len(idx)]
+            if not inner:
+                continue
+            a_in, b_in = min(inner, key=lambda ab: ab[1] - ab[0])
+            if not any(a_ < a_in and b_in < b_ for a_, b_ in loops):
+                continue   # not nested: nothing can be hoisted out of it
+            for i in idx:
+                if not (a_in <= i <= b_in) and any(a_ <= i <= b_ for a_, b_ in loops):
+                    final[i] = (ename, False)
         reg = {}
         unmapped = 0
         instr = []   # (byte offset, region key or None = cold, issue weight)

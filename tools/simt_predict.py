@@ -61,12 +61,13 @@ def find(costs_all, pattern):
     raise KeyError(pattern)
 
 
-def divloop_warps(mode, T):
+def divloop_warps(mode, T, V=None):
     c = I.C1
+    V = c.advance_unroll if V is None else V
     want = oracle.divloop_wants(0, c.n_threads, c.iters, I.PRIMARY_SEED, c.p_u32)
     for w in range(0, c.n_threads, 32):
         ww = want[w:w + 32]
-        yield oracle.ws_divloop(ww, mode, T), len(ww)
+        yield oracle.ws_divloop(ww, mode, T, V=V if mode == oracle.SPEC_LOOP else 1), len(ww)
 
 
 def commoncall_warps(mode):

@@ -89,7 +89,7 @@ if "divloop" in a.what:
     c = I.C1
     res = []
     for b in blocks:
-        w = sr.divloop_workload(c.p_u32, c.fma_count, block=b)
+        w = sr.divloop_workload(c.p_u32, c.fma_count, block=b, advance=a.unroll)
         ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
             def run():
