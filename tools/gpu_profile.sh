@@ -7,6 +7,9 @@ TAG=${1:-r01}
 O=gpurun_out
 mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()"
+# SASS hashes of the kernels this run measures (tools/summarize_ncu.py stores them with the
+# measurements, so a later local rebuild cannot be mistaken for the measured code)
+python -c "import json,sys; sys.path.insert(0,'tools'); import sass_regions as S; json.dump(S.kernel_hashes('divloop_|commoncall_|mcml_|pt_|rs_'), open('$O/sass_hashes_$TAG.json','w'))"
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > $O/gpu_$TAG.txt
 if [ "$2" != "quick" ]; then
   timeout 1200 python -m pytest tests -m gpu -q > $O/tests_$TAG.log 2>&1; tail -3 $O/tests_$TAG.log

@@ -108,7 +108,12 @@ def main():
                      " libsr built from this commit")
     sys.path.insert(0, os.path.join(ROOT, "tools"))
     import sass_regions
-    hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_|pt_|rs_")
+    hpath = os.path.join(OUT, f"sass_hashes_{tag}.json")
+    if os.path.exists(hpath):   # hashed on the GPU box, from the build it measured
+        hashes = json.load(open(hpath))
+    else:
+        print("warning: no box-side SASS hashes; hashing the local build", file=sys.stderr)
+        hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_|pt_|rs_")
     for lab, r in js.items():
         if isinstance(r, dict):
             mangled = [k for k in hashes if mangle_match(r["kernel"], k)]
