@@ -134,7 +134,9 @@ typedef struct {
   int32_t kind;            /* sr_workload_kind                                   */
   uint32_t flags;          /* SR_F_*                                             */
   uint64_t task_offset;    /* global id of this caller's first task (sharding)  */
-  uint32_t block_threads;  /* CTA size, multiple of 32 in [32,1024]; 0 = default */
+  uint32_t block_threads;  /* CTA size, multiple of 32 in [32, bound]; 0 = default.
+                              bound: MCML 640, PATHTRACE 128, RSBENCH 256, else 1024
+                              (the kernels' __launch_bounds__)                   */
   uint32_t grid_ctas;      /* dynamic-claiming kernels: CTAs; 0 = fill the GPU   */
   sr_divloop_params divloop;
   sr_commoncall_params commoncall;
@@ -158,7 +160,11 @@ SR_API int sr_init(int device, void* cuda_stream, void* workspace_dev, size_t wo
  *   SR_T_COUNTERS   uint64[16] workload counters (see sr_counter_names in DESIGN.md)
  *   SR_T_SCHED      per warp: uint32[8] schedule counters (only with SR_F_SCHED):
  *                   {rounds, release rounds, common-code lane-executions,
- *                    advance rounds, prolog lane-executions, 0, 0, 0}
+ *                    advance rounds, lanes taking part in advance rounds
+ *                    (sum of popc(R); with DIVLOOP advance_unroll > 1 a lane
+ *                    may run several prologs in one such round), 0, 0, 0};
+ *                   one record per launched warp (warps past n_threads are
+ *                   not written)
  *   SR_T_SCRATCH    internal (claim counters)
  * GRID and COUNTERS are contiguous so a multi-GPU caller can reduce them
  * in place as int64 (two's-complement addition = uint64 addition mod 2^64). */
@@ -173,8 +179,12 @@ SR_API int sr_workspace_region(const sr_workload* w, uint64_t n_threads, int wha
  * per pixel).  threshold: soft-barrier size T in [1,32], 0 = 32 ("wait for
  * all", Fig. 1(b)); ignored for SR_PDOM; must be 0 or 32 for SR_SPEC_CALL.
  * SR_SPEC_CALL is valid only for COMMONCALL; SR_SPEC_LOOP only for DIVLOOP,
- * MCML, PATHTRACE.  Zeroes the output regions, then enqueues the kernel(s);
- * does not synchronize.  Every output bit is a function of (workload params,
+ * MCML, PATHTRACE, RSBENCH.  Zeroes the output regions, then enqueues the
+ * kernel(s); does not synchronize, so a run can be captured in a CUDA graph.
+ * (PATHTRACE: the scene header is known on the host when sr_scene_build wrote
+ * the image in this process; an image copied in by the caller is read once,
+ * synchronously on the context stream -- SR_E_CUDA if that stream is
+ * capturing -- and remembered afterwards.)  Every output bit is a function of (workload params,
  * seed, task ids) only -- never of mode, threshold, block size, grid size or
  * GPU count.
  * Errors: SR_E_STATE before sr_init; SR_E_INVALID (n_threads == 0,

@@ -369,3 +369,49 @@ def pt_closest(scene, o, d):
     i = lib().or_pt_closest(scene.tris, scene.n_tris, _p(o, C.c_float), _p(d, C.c_float),
                             C.byref(t))
     return int(i), t.value
+
+
+# ---------------------------------------------------------------- step building blocks (pins)
+def mcml_step_length(mut, u0):
+    """or_mcml_step_length over an array of Philox words u0."""
+    u = np.ascontiguousarray(u0, np.uint32)
+    out = np.empty(u.size, np.float32)
+    L = lib()
+    L.or_mcml_eval_batch.argtypes = [C.c_int, C.c_float, C.POINTER(C.c_uint32),
+                                     C.POINTER(C.c_float), C.c_uint64]
+    L.or_mcml_eval_batch(0, mut, _p(u, C.c_uint32), _p(out, C.c_float), u.size)
+    return out
+
+
+def mcml_hg_cost(g, u1):
+    """or_mcml_hg_cost(g, U01(u1)) over an array of Philox words u1."""
+    u = np.ascontiguousarray(u1, np.uint32)
+    out = np.empty(u.size, np.float32)
+    L = lib()
+    L.or_mcml_eval_batch.argtypes = [C.c_int, C.c_float, C.POINTER(C.c_uint32),
+                                     C.POINTER(C.c_float), C.c_uint64]
+    L.or_mcml_eval_batch(1, g, _p(u, C.c_uint32), _p(out, C.c_float), u.size)
+    return out
+
+
+def mcml_spin(cost, xi_psi, u):
+    L = lib()
+    fp = C.POINTER(C.c_float)
+    L.or_mcml_spin.argtypes = [C.c_float, C.c_float, fp, fp]
+    ui = np.ascontiguousarray(u, np.float32)
+    uo = np.zeros(3, np.float32)
+    L.or_mcml_spin(cost, xi_psi, _p(ui, C.c_float), _p(uo, C.c_float))
+    return uo
+
+
+def pt_scatter(kind, ior, d, ng, u):
+    """or_pt_scatter: the direction half of one path-tracer bounce."""
+    L = lib()
+    fp = C.POINTER(C.c_float)
+    L.or_pt_scatter.argtypes = [C.c_uint32, C.c_float, fp, fp, C.POINTER(C.c_uint32), fp]
+    di = np.ascontiguousarray(d, np.float32); ni = np.ascontiguousarray(ng, np.float32)
+    uu = np.ascontiguousarray(u, np.uint32)
+    do = np.zeros(3, np.float32)
+    L.or_pt_scatter(kind, ior, _p(di, C.c_float), _p(ni, C.c_float), _p(uu, C.c_uint32),
+                    _p(do, C.c_float))
+    return do

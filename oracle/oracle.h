@@ -102,6 +102,11 @@ uint64_t or_mcml_events_batch(const or_mcml_params* p, uint64_t id0, uint64_t co
 float or_mcml_fresnel(float ni, float nt, float ca1, float* ca2);
 /* Rsp as defined in mcml.c (specular reflectance at launch) */
 float or_mcml_rsp(const or_mcml_params* p);
+/* the step's building blocks, exactly as step() uses them (pins in tests/) */
+float or_mcml_step_length(float mut, uint32_t u0);   /* -ln(U01c(u0)) / mu_t   */
+float or_mcml_hg_cost(float g, float xi);            /* HG cos(theta)          */
+void or_mcml_spin(float cost, float xi_psi, const float u_in[3], float u_out[3]);
+void or_mcml_eval_batch(int fn, float p, const uint32_t* u, float* out, uint64_t n);
 
 /* ---- pathtrace.c : config 4, path tracer with brute-force closest hit. */
 typedef struct {
@@ -115,6 +120,9 @@ typedef struct {
 /* closest hit over all triangles (t > 1e-4; ties -> smaller index); -1 = miss */
 int64_t or_pt_closest(const float* tris, uint32_t n_tris, const float o[3], const float d[3],
                       float* t_best);
+/* the direction half of one bounce (material kind 0/1/2; see pathtrace.c) */
+void or_pt_scatter(uint32_t kind, float ior, const float d_in[3], const float ng_in[3],
+                   const uint32_t u[4], float d_out[3]);
 /* rgb[3k..3k+2] = sum over the spp samples of pixel pixels[k] (all pixels
  * 0..n_pixels-1 when pixels == NULL); counters[0] += paths, [1] += rays. */
 void or_pt_render(const or_pt_scene* sc, uint32_t width, uint32_t height, uint32_t spp,

@@ -90,6 +90,54 @@ static void draw(uint32_t event, uint64_t q, uint64_t seed, uint32_t u[4]) {
   or_philox4x32_10(ctr, key, u);
 }
 
+/* The direction half of a bounce (reading R7), after the hit: ng = the unit
+ * geometric normal of the hit triangle, d = the incoming unit direction, u =
+ * the bounce's Philox draw, ior = the material's index.  The shading normal n
+ * is ng flipped to face the incoming ray; entering = the ray arrives on ng's
+ * side.
+ *   kind 0 diffuse:    cosine-weighted about n (Malley: a uniform point of the
+ *                      unit disk, r = sqrt(U01(u0)), phi = 2 pi U01(u1), lifted
+ *                      to the hemisphere), in the Duff et al. basis of n;
+ *   kind 1 mirror:     d - 2 (d.n) n;
+ *   kind 2 dielectric: eta = 1/ior entering, ior leaving; Schlick reflectance
+ *                      F = r0 + (1 - r0)(1 - cos_i)^5, r0 = ((1-ior)/(1+ior))^2;
+ *                      reflect if total internal reflection (k < 0) or
+ *                      U01(u2) < F, else refract: eta d + (eta cos_i - sqrt(k)) n.
+ * Exported so the tests can check each branch against float64 geometry. */
+void or_pt_scatter(uint32_t kind, float ior, const float d_in[3], const float ng_in[3],
+                   const uint32_t u[4], float d_out[3]) {
+  v3 d = mk(d_in[0], d_in[1], d_in[2]), ng = mk(ng_in[0], ng_in[1], ng_in[2]);
+  float cosd = dot(ng, d);
+  int entering = cosd < 0.0f;
+  v3 n = entering ? ng : scl(ng, -1.0f);                /* faces the incoming ray */
+  if (kind == 0u) {                                     /* diffuse: cosine-weighted */
+    float r1 = or_u01(u[0]);
+    float rr = sqrtf(r1);
+    float sp, cp;
+    or_sr_sincos2pif(or_u01(u[1]), &sp, &cp);
+    float lx = rr * cp, ly = rr * sp, lz = sqrtf(1.0f - r1);
+    v3 t1, t2;
+    onb(n, &t1, &t2);
+    d = add(add(scl(t1, lx), scl(t2, ly)), scl(n, lz));
+  } else if (kind == 1u) {                              /* mirror */
+    d = sub(d, scl(n, 2.0f * dot(d, n)));
+  } else {                                              /* dielectric */
+    float eta = entering ? 1.0f / ior : ior;
+    float cosi = -dot(d, n);
+    float k = 1.0f - eta * eta * (1.0f - cosi * cosi);
+    float r0 = (1.0f - ior) / (1.0f + ior);
+    r0 = r0 * r0;
+    float c5 = 1.0f - cosi;
+    float fr = r0 + (1.0f - r0) * (c5 * c5 * c5 * c5 * c5);
+    if (k < 0.0f || or_u01(u[2]) < fr) {
+      d = sub(d, scl(n, 2.0f * dot(d, n)));             /* reflect */
+    } else {
+      d = add(scl(d, eta), scl(n, eta * cosi - sqrtf(k)));  /* refract */
+    }
+  }
+  d_out[0] = d.x; d_out[1] = d.y; d_out[2] = d.z;
+}
+
 /* One path of sample id q for pixel (px, py).  rgb += radiance is done by
  * the caller; counters: [0] bounces (rays traced). */
 static v3 trace_path(const or_pt_scene* sc, uint32_t px, uint32_t py, uint64_t q, uint64_t seed,
@@ -122,40 +170,12 @@ static v3 trace_path(const or_pt_scene* sc, uint32_t px, uint32_t py, uint64_t q
     v3 e1 = sub(mk(tri[3], tri[4], tri[5]), v0);
     v3 e2 = sub(mk(tri[6], tri[7], tri[8]), v0);
     v3 ng = normalize(cross(e1, e2));
-    float cosd = dot(ng, d);
-    int entering = cosd < 0.0f;
-    v3 n = entering ? ng : scl(ng, -1.0f);                /* faces the incoming ray */
     v3 p = add(o, scl(d, t));
     draw(b + 1u, q, seed, u);
-    if (kind == 0u) {                                     /* diffuse: cosine-weighted */
-      float r1 = or_u01(u[0]);
-      float rr = sqrtf(r1);
-      float sp, cp;
-      or_sr_sincos2pif(or_u01(u[1]), &sp, &cp);
-      float lx = rr * cp, ly = rr * sp, lz = sqrtf(1.0f - r1);
-      v3 t1, t2;
-      onb(n, &t1, &t2);
-      d = add(add(scl(t1, lx), scl(t2, ly)), scl(n, lz));
-      thr = mk(thr.x * m[1], thr.y * m[2], thr.z * m[3]);
-    } else if (kind == 1u) {                              /* mirror */
-      d = sub(d, scl(n, 2.0f * dot(d, n)));
-      thr = mk(thr.x * m[1], thr.y * m[2], thr.z * m[3]);
-    } else {                                              /* dielectric */
-      float ior = m[7];
-      float eta = entering ? 1.0f / ior : ior;
-      float cosi = -dot(d, n);
-      float k = 1.0f - eta * eta * (1.0f - cosi * cosi);
-      float r0 = (1.0f - ior) / (1.0f + ior);
-      r0 = r0 * r0;
-      float c5 = 1.0f - cosi;
-      float fr = r0 + (1.0f - r0) * (c5 * c5 * c5 * c5 * c5);
-      if (k < 0.0f || or_u01(u[2]) < fr) {
-        d = sub(d, scl(n, 2.0f * dot(d, n)));             /* reflect */
-      } else {
-        d = add(scl(d, eta), scl(n, eta * cosi - sqrtf(k)));  /* refract */
-      }
-      thr = mk(thr.x * m[1], thr.y * m[2], thr.z * m[3]);
-    }
+    float dd_in[3] = {d.x, d.y, d.z}, ng3[3] = {ng.x, ng.y, ng.z}, dout[3];
+    or_pt_scatter(kind, m[7], dd_in, ng3, u, dout);
+    d = mk(dout[0], dout[1], dout[2]);
+    thr = mk(thr.x * m[1], thr.y * m[2], thr.z * m[3]);
     o = p;
     if (b >= 3u) {                                        /* Russian roulette */
       float pm = fmaxf(thr.x, fmaxf(thr.y, thr.z));

@@ -314,6 +314,7 @@ static int build_scene(const char* fn, bool to_device, const float* tris, const 
     const cudaError_t e = cudaMemcpy(dst, img.data(), h.bytes, cudaMemcpyHostToDevice);
     if (e != cudaSuccess)
       return set_error(SR_E_CUDA, std::string(fn) + ": cudaMemcpy: " + cudaGetErrorString(e));
+    register_scene(dst, &h);
   } else {
     std::memcpy(dst, img.data(), h.bytes);
   }

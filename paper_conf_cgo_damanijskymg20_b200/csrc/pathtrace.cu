@@ -29,6 +29,11 @@
 // the brute-force closest hit, ties to the smaller triangle id; conservative
 // padded-box slab test) + material shading, operation for operation as
 // oracle/pathtrace.c (reading R7).
+#include <cstring>
+#include <mutex>
+#include <utility>
+#include <vector>
+
 #include "pt_scene.h"
 #include "sr_device.cuh"
 #include "sr_internal.h"
@@ -435,7 +440,7 @@ __device__ __forceinline__ void bounce(const PtArgs& a, Path& p, Trav& tr, Stats
 }
 
 template <bool SCHED>
-__global__ void __launch_bounds__(128, SR_PT_MINB_PDOM) pt_pdom(const PtArgs a) {
+__global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_PDOM) pt_pdom(const PtArgs a) {
   const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = g < a.n;
@@ -478,7 +483,7 @@ __global__ void __launch_bounds__(128, SR_PT_MINB_PDOM) pt_pdom(const PtArgs a) 
 // count (nodes per ray) varies most.  SPLIT (with NODE): the node visit's
 // leaf triangle tests become their own region (trav_node / trav_leaf).
 template <bool SCHED, bool NODE, bool SPLIT = false>
-__global__ void __launch_bounds__(128, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) {
+__global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) {
   const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = g < a.n;
@@ -610,9 +615,47 @@ std::string check_pathtrace(const sr_pathtrace_params& p, uint64_t n_threads) {
 
 size_t pathtrace_perthread_bytes(uint64_t n) { return 12 * n; }
 
-static cudaError_t read_header(const void* scene, PtHeader& h) {
-  cudaError_t e = cudaMemcpy(&h, scene, sizeof h, cudaMemcpyDeviceToHost);
-  if (e != cudaSuccess) return e;
+// Scene headers known on the host: sr_scene_build registers the header of every
+// image it writes, so a run needs no device->host read of it (sr_run stays
+// stream-ordered and capturable in a CUDA graph).  An image the library did not
+// write in this process (e.g. one built with sr_scene_build_host and copied by
+// the caller) is read once -- a synchronous copy on the context stream, refused
+// during stream capture -- and then registered too.  An entry stays valid while
+// the caller's buffer holds that image.
+namespace {
+std::mutex g_scene_mu;
+std::vector<std::pair<const void*, PtHeader>> g_scenes;
+}  // namespace
+
+void register_scene(const void* dev, const void* header) {
+  std::lock_guard<std::mutex> lk(g_scene_mu);
+  PtHeader h;
+  std::memcpy(&h, header, sizeof h);
+  for (auto& e : g_scenes)
+    if (e.first == dev) { e.second = h; return; }
+  g_scenes.emplace_back(dev, h);
+}
+
+static cudaError_t read_header(cudaStream_t st, const void* scene, PtHeader& h) {
+  bool known = false;
+  {
+    std::lock_guard<std::mutex> lk(g_scene_mu);
+    for (const auto& e : g_scenes)
+      if (e.first == scene) { h = e.second; known = true; break; }
+  }
+  if (!known) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    cudaError_t e = cudaStreamIsCapturing(st, &cs);
+    if (e != cudaSuccess) return e;
+    if (cs != cudaStreamCaptureStatusNone) {
+      set_launch_note("scene_dev was not written by sr_scene_build in this process; its header "
+                      "cannot be read during stream capture");
+      return cudaErrorInvalidValue;
+    }
+    e = cudaMemcpyAsync(&h, scene, sizeof h, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return e;
+  }
   if (h.magic != kPtMagic) {
     set_launch_note("scene_dev does not hold an sr_scene_build image");
     return cudaErrorInvalidValue;
@@ -622,13 +665,14 @@ static cudaError_t read_header(const void* scene, PtHeader& h) {
                     " entries, more than " + std::to_string(kMaxStack));
     return cudaErrorInvalidValue;
   }
+  if (!known) register_scene(scene, &h);
   return cudaSuccess;
 }
 
 cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t n, uint32_t iters,
                              uint64_t seed, int mode, uint32_t T) {
   PtHeader h;
-  cudaError_t e = read_header(w.pathtrace.scene_dev, h);
+  cudaError_t e = read_header(c.stream, w.pathtrace.scene_dev, h);
   if (e != cudaSuccess) return e;
   if (h.bytes > w.pathtrace.scene_bytes) {
     set_launch_note("pathtrace.scene_bytes is smaller than the scene image");
@@ -690,7 +734,7 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
 cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* rays, int64_t* hit,
                             float* t, uint64_t n) {
   PtHeader h;
-  cudaError_t e = read_header(scene, h);
+  cudaError_t e = read_header(st, scene, h);
   if (e != cudaSuccess) return e;
   PtArgs a = base_args(scene);
   a.nodes = reinterpret_cast<const PtNode*>(a.scene + h.off_nodes);
@@ -701,9 +745,18 @@ cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* ray
   a.q_hit = hit;
   a.q_t = t;
   a.stack_cap = h.stack_need > 0 ? h.stack_need : 1u;
-  const unsigned grid = (unsigned)((n + 127) / 128);
-  record_launch(grid, 128, 0);
-  if (n) pt_query<<<grid, 128, a.stack_cap * 128 * sizeof(int32_t), st>>>(a);
+  const uint64_t grid = (n + 127) / 128;
+  if (grid > 0x7fffffffull) {
+    set_launch_note("too many rays for one launch");
+    return cudaErrorInvalidValue;
+  }
+  const size_t smem = (size_t)a.stack_cap * 128 * sizeof(int32_t);
+  if (smem > 48 * 1024) {
+    e = cudaFuncSetAttribute(pt_query, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+  }
+  record_launch((uint32_t)grid, 128, (uint32_t)smem);
+  if (n) pt_query<<<(unsigned)grid, 128, smem, st>>>(a);
   return cudaGetLastError();
 }
 

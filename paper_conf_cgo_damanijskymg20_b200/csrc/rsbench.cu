@@ -72,7 +72,7 @@ __device__ __forceinline__ void finish(const RsArgs& a, uint64_t g, bool valid, 
   const uint32_t tot = __reduce_add_sync(kFull, valid ? nucs : 0u);
   if (lane_id() == 0) {
     atomicAdd(a.counters, (unsigned long long)tot);
-    if (a.sched) {
+    if (a.sched && (g & ~31ull) < a.n) {
       uint4* p = reinterpret_cast<uint4*>(a.sched + (g >> 5) * kSchedWords);
       p[0] = make_uint4(rounds, rel, rel_lanes, adv);
       p[1] = make_uint4(adv_lanes, 0u, 0u, 0u);
@@ -81,7 +81,7 @@ __device__ __forceinline__ void finish(const RsArgs& a, uint64_t g, bool valid, 
 }
 
 template <int ROUNDS, int PROLOG, bool SCHED>
-__global__ void __launch_bounds__(256) rs_pdom(const RsArgs a) {
+__global__ void __launch_bounds__(SR_RS_MAXT) rs_pdom(const RsArgs a) {
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
   const bool valid = g < a.n;
   const uint64_t t = a.t0 + g;
@@ -114,7 +114,7 @@ __global__ void __launch_bounds__(256) rs_pdom(const RsArgs a) {
 }  // @sr-region END
 
 template <int ROUNDS, int PROLOG, bool SCHED>
-__global__ void __launch_bounds__(256) rs_spec(const RsArgs a) {
+__global__ void __launch_bounds__(SR_RS_MAXT) rs_spec(const RsArgs a) {
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
   const bool valid = g < a.n;
   const uint64_t t = a.t0 + g;

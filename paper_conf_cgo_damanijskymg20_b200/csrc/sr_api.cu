@@ -45,12 +45,25 @@ int fail_cuda(cudaError_t e, const char* where) {
 }
 size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
 
+// __launch_bounds__ of each workload's kernels
+uint32_t max_block(int kind) {
+  switch (kind) {
+    case SR_WL_MCML: return SR_MCML_MAXT;
+    case SR_WL_PATHTRACE: return SR_PT_MAXT;
+    case SR_WL_RSBENCH: return SR_RS_MAXT;
+    default: return 1024;
+  }
+}
+
 std::string check_workload(const sr_workload* w, uint64_t n_threads) {
   if (!w) return "workload is NULL";
   if (n_threads == 0) return "n_threads must be >= 1";
   if (w->block_threads != 0 &&
       (w->block_threads % 32 != 0 || w->block_threads < 32 || w->block_threads > 1024))
     return "block_threads must be 0 or a multiple of 32 in [32, 1024]";
+  if (w->block_threads > max_block(w->kind))
+    return "block_threads exceeds this workload's kernels' launch bound (" +
+           std::to_string(max_block(w->kind)) + ")";
   if (w->flags & ~(SR_F_SCHED | SR_F_STATIC | SR_F_COARSE | SR_F_NOSPLIT)) return "unknown flags";
   switch (w->kind) {
     case SR_WL_DIVLOOP:
@@ -110,8 +123,10 @@ Layout layout_of(const sr_workload& w, uint64_t n) {
     default: break;
   }
   const uint32_t block = default_block(w);
-  // schedule counters: one record per warp of the largest grid any kernel uses
-  uint64_t warps = (n + 31) / 32;
+  // schedule counters: one record per launched warp of the largest grid any kernel
+  // uses (a partial last CTA launches whole warps past n; kernels also skip the
+  // record of a warp whose first thread is >= n)
+  uint64_t warps = ((n + block - 1) / block) * (block / 32);
   if (w.kind == SR_WL_MCML || w.kind == SR_WL_PATHTRACE) {
     const uint64_t gw = ((n + block - 1) / block) * (block / 32);
     const uint64_t dyn = (uint64_t)2048 * 1024 / 32;  // >= any persistent grid (148 SMs x 2048)

@@ -17,6 +17,10 @@ namespace sr {
 #define SR_MCML_MAXT 640
 #endif
 
+// CTA-size launch bounds of the path-tracer and RSBench kernels
+#define SR_PT_MAXT 128
+#define SR_RS_MAXT 256
+
 constexpr int kCounters = 16;
 constexpr int kSchedWords = 8;  // uint32 per warp
 
@@ -69,5 +73,7 @@ cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* ray
 std::string check_mcml(const sr_mcml_params& p);
 std::string check_pathtrace(const sr_pathtrace_params& p, uint64_t n_threads);
 size_t pathtrace_perthread_bytes(uint64_t n_threads);
+// Remember the header (a PtHeader, 128 bytes) of a scene image written to `dev`.
+void register_scene(const void* dev, const void* header);
 
 }  // namespace sr

@@ -280,6 +280,9 @@ class Context:
     def ensure(self, nbytes: int):
         if self.workspace.numel() < nbytes:
             import torch
+            # kernels enqueued by libsr on self.stream may still use the old block;
+            # the caching allocator could hand it out again once it is dropped
+            self.stream.synchronize()
             self.workspace = torch.empty(nbytes, dtype=torch.uint8, device=f"cuda:{self.device}")
             sr_init(self.device, self.stream.cuda_stream, self.workspace.data_ptr(), nbytes)
 
