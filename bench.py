@@ -6,10 +6,12 @@ JSON line on rank 0.  For N > 1 it is launched under torch.distributed.run, one
 process per GPU, NCCL.
 
 Headline workload: Monte Carlo photon transport in the
-3-layer slab (BASELINE.json configs[2]: 10^7 photons per GPU), Loop Merge
-(SR_SPEC_LOOP, T=32) -- one step = one sr_run over the rank's photon shard plus,
-for N > 1, one NCCL all-reduce of the integer tallies (configs[4] is this run
-weak-scaled: N x 10^7 photons).  The PDOM kernel is timed the same way
+3-layer slab, Loop Merge (SR_SPEC_LOOP, T=32) -- one step = one sr_run over the
+rank's photon shard plus, for N > 1, one NCCL all-reduce of the integer tallies.
+N = 1: configs[2] (10^7 photons).  N > 1: configs[4], 10^9 photons in total split
+over the N ranks (strong scaling); rank 0 also times the whole 10^9 alone (t_1 of
+E_N = t_1/(N t_N)) and the line carries the weak-scaled 10^7-per-rank numbers
+under "scaling_detail".  The PDOM kernel is timed the same way
 ("pdom" key).  At N = 1 the two microbenchmarks (configs[0], configs[1]) are
 timed too ("configs" key), PDOM vs SPEC.
 
@@ -46,7 +48,15 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--threshold", type=int, default=32)
     ap.add_argument("--photons-per-gpu", type=int, default=0,
-                    help="override the per-rank photon count (default: configs[2] = 10^7)")
+                    help="override the per-rank photon count of N = 1 / weak runs "
+                         "(default: configs[2] = 10^7)")
+    ap.add_argument("--total-photons", type=int, default=0,
+                    help="N > 1 strong scaling: photons of the whole job (default: configs[4] "
+                         "= 10^9)")
+    ap.add_argument("--scaling", default="auto", choices=["auto", "strong", "weak"],
+                    help="N > 1: strong (configs[4], default) or weak (10^7 per rank)")
+    ap.add_argument("--t1-steps", type=int, default=2,
+                    help="N > 1: timed single-GPU runs of the whole job (t_1 of E_N)")
     ap.add_argument("--block", type=int, default=0, help="MCML CTA size (0 = library default)")
     ap.add_argument("--unroll", type=int, default=0,
                     help="MCML steps per release (0 = inputs.C3.merge_unroll)")
@@ -265,25 +275,45 @@ def main():
     sr.load()  # raises if libsr.so is missing: no fallback
 
     m = I.C3
-    per_rank = args.photons_per_gpu or m.n_photons
     iters = m.iters
-    nt = (per_rank + iters - 1) // iters
-    per_rank = nt * iters
     T = args.threshold
-    w = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap,
-                         task_offset=P.task_offset_of(rank, per_rank), block=args.block,
-                         unroll=args.unroll if args.unroll else m.merge_unroll)
+    unroll = args.unroll if args.unroll else m.merge_unroll
+    # N = 1: configs[2] (10^7 photons).  N > 1: configs[4] -- a fixed total of
+    # 10^9 photons split over the ranks (strong scaling),
+    # unless --scaling weak keeps 10^7 (or --photons-per-gpu) per rank.
+    strong = ws_n > 1 and args.scaling != "weak"
+    if strong:
+        total = args.total_photons or I.C5_TOTAL_PHOTONS
+        nt_total = (total + iters - 1) // iters
+        lane0, nt = P.split_even(nt_total, ws_n, rank)
+        total = nt_total * iters
+        offset = lane0 * iters
+    else:
+        per_rank = args.photons_per_gpu or m.n_photons
+        nt = (per_rank + iters - 1) // iters
+        total = nt * iters * ws_n
+        offset = P.task_offset_of(rank, nt * iters)
+    per_rank = nt * iters
+
+    def mc_workload(task_offset, flags=0):
+        return sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz,
+                                m.step_cap, task_offset=task_offset, block=args.block,
+                                unroll=unroll, flags=flags)
+
+    w = mc_workload(offset)
     nbytes = sr.sr_workspace_bytes(w, nt)
     ctx = sr.Context.create(local, nbytes, stream)
     off, tb = sr.sr_workspace_region(w, nt, sr.T_GRID)
     _, cb = sr.sr_workspace_region(w, nt, sr.T_COUNTERS)
-    tallies = ctx.workspace[off:off + tb + cb].view(torch.int64)  # GRID + COUNTERS, contiguous
     barrier = (lambda: dist.barrier()) if ws_n > 1 else None
     timer = Timer(torch, stream)
 
+    def tallies_view():   # GRID + COUNTERS, contiguous (re-taken: ctx.ensure may reallocate)
+        return ctx.workspace[off:off + tb + cb].view(torch.int64)
+
     def step(mode, thr):
         sr.sr_run(w, nt, iters, I.PRIMARY_SEED, mode, thr)
-        P.allreduce_tallies(tallies, stream=stream)   # no-op at N = 1
+        P.allreduce_tallies(tallies_view(), stream=stream)   # no-op at N = 1
 
     # device-timed region, SPEC (headline) with clocks sampled during it
     with ClockSampler(local) as clk:
@@ -307,20 +337,18 @@ def main():
     coll = None
     if ws_n > 1:
         def allreduce_only():
-            P.allreduce_tallies(tallies, stream=stream)
+            P.allreduce_tallies(tallies_view(), stream=stream)
         ms_ar = timer.time_steps(allreduce_only, args.steps, args.warmup, barrier)
         t_ar = max_over_ranks(statistics.mean(ms_ar))
         coll = {"op": f"all_reduce(SUM) int64, {args.dist_backend}", "bytes": tb + cb,
                 "ms": t_ar, "share_of_step": t_ar / t_spec}
     t_pdom = max_over_ranks(statistics.mean(ms_pdom))
-    total = per_rank * ws_n
     value = total / (t_spec * 1e-3)
     pdom_value = total / (t_pdom * 1e-3)
 
     # end to end through the public API: sr_run + (all-reduce) + sr_tally into
     # pinned host memory, host wall clock per step, max over ranks
     host = torch.empty(tb + cb, dtype=torch.uint8, pin_memory=True)
-    h2d = 0
     import ctypes
     h2d = ctypes.sizeof(sr.Workload)   # the step's inputs: the workload descriptor
     e2e_ms = []
@@ -343,10 +371,10 @@ def main():
     # schedule-level efficiency of the common code (instrumented kernels, outside timing)
     def region_eff(mode, thr):
         wi = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz,
-                              m.step_cap, task_offset=P.task_offset_of(rank, per_rank),
+                              m.step_cap, task_offset=offset,
                               flags=sr.F_SCHED)   # U = 1: lanes per merged-loop iteration
-        ctx.ensure(sr.sr_workspace_bytes(wi, nt))
         ni = min(nt, 32768)
+        ctx.ensure(sr.sr_workspace_bytes(wi, ni))
         sr.sr_run(wi, ni, iters, I.PRIMARY_SEED, mode, thr)
         s = ctx.region(wi, ni, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS)
         s = s.cpu().numpy().astype("int64")
@@ -356,24 +384,49 @@ def main():
     eff_spec = region_eff(sr.SPEC_LOOP, T)
     eff_pdom = region_eff(sr.PDOM, 0)
 
-    # N > 1: the whole job's photons once more on rank 0 in ONE launch (ids
-    # [0, N x per_rank), the union of the shards) -- the all-reduced tallies of
-    # the last step must equal it bit for bit (SURVEY.md Sec. 8(e) invariant)
+    # N > 1: the whole job once more on rank 0 alone, in ONE launch per step over
+    # every photon id [0, total): (i) the all-reduced tallies of the sharded run
+    # must equal it bit for bit (SURVEY.md Sec. 8(e) invariant); (ii) strong
+    # scaling: its device time is t_1 of E_N = t_1 / (N t_N)
     same_as_one_gpu = None
+    scaling = None
     if ws_n > 1:
+        t1 = None
         if rank == 0:
-            w_all = sr.mcml_workload(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz,
-                                     m.step_cap, task_offset=P.task_offset_of(0, per_rank),
-                                     block=args.block,
-                                     unroll=args.unroll if args.unroll else m.merge_unroll)
-            nt_all = nt * ws_n
+            w_all = mc_workload(0)
+            nt_all = total // iters
             ctx.ensure(sr.sr_workspace_bytes(w_all, nt_all))
-            sr.sr_run(w_all, nt_all, iters, I.PRIMARY_SEED, sr.SPEC_LOOP, T)
+            ms_1 = timer.time_steps(
+                lambda: sr.sr_run(w_all, nt_all, iters, I.PRIMARY_SEED, sr.SPEC_LOOP, T),
+                args.t1_steps, 1)
+            t1 = statistics.mean(ms_1)
             ref = torch.empty(tb + cb, dtype=torch.uint8, pin_memory=True)
             sr.sr_tally(sr.T_GRID, ref.data_ptr(), tb)
             sr.sr_tally(sr.T_COUNTERS, ref.data_ptr() + tb, cb)
             same_as_one_gpu = bool(torch.equal(ref, host))
         dist.barrier()
+        # the other reading of configs[4]: a fixed 10^7 photons per rank (weak)
+        nt_w = m.n_photons // iters
+        w_weak = mc_workload(P.task_offset_of(rank, nt_w * iters))
+        ctx.ensure(sr.sr_workspace_bytes(w_weak, nt_w))
+
+        def weak_step():
+            sr.sr_run(w_weak, nt_w, iters, I.PRIMARY_SEED, sr.SPEC_LOOP, T)
+            P.allreduce_tallies(tallies_view(), stream=stream)
+        t_weak = max_over_ranks(statistics.mean(
+            timer.time_steps(weak_step, args.steps, args.warmup, barrier)))
+        if rank == 0:
+            v1 = total / (t1 * 1e-3)
+            scaling = {
+                "kind": "strong" if strong else "weak",
+                "t1_ms": t1, "t1_value": v1,
+                "t1_basis": f"rank 0 alone, all {total} photons in one launch per step, "
+                            f"{args.t1_steps} timed steps",
+                "efficiency": (t1 / (ws_n * t_spec)) if strong else value / (ws_n * v1),
+                "efficiency_basis": ("E_N = t_1 / (N t_N), SURVEY.md Sec. 8(e)" if strong else
+                                     "value_N / (N x t1_value)"),
+                "weak": {"photons_per_gpu": nt_w * iters, "ms_per_step": t_weak,
+                         "value": ws_n * nt_w * iters / (t_weak * 1e-3)}}
 
     peaks = load_json(PEAKS_FILE) or {}
     consts = load_json(PROFILE_CONST) or {}
@@ -393,11 +446,18 @@ def main():
                   "kernel": "mcml_spec",
                   "peak_basis": f"592 SMSPs x 32 lanes x {f_mhz:.0f} MHz (sm_max_mhz of measured)",
                   "work_basis": "profiles/work_per_unit.json: PDOM thread-inst per photon step (ncu)"}
+        if strong:
+            workload_name = f"mcml-3layer configs[4]: {total} photons sharded over {ws_n} GPUs"
+        elif ws_n > 1:
+            workload_name = f"mcml-3layer configs[2] shape, {per_rank} photons per GPU (weak)"
+        else:
+            workload_name = f"mcml-3layer configs[2]: {total} photons"
         result = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws_n, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t_spec, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": "mcml-3layer (configs[2] per GPU; N GPUs = configs[4] weak-scaled)",
+            "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic",
+            "config": {"workload": workload_name, "total_photons": total,
                        "photons_per_gpu": per_rank, "lanes": nt, "photons_per_lane": iters,
                        "threshold": T, "mode": "SPEC_LOOP", "seed": I.PRIMARY_SEED,
                        "merge_unroll": args.unroll if args.unroll else m.merge_unroll,
@@ -417,6 +477,7 @@ def main():
             "roofline": rl,
             "collective": coll,
             "tallies_equal_single_gpu_run": same_as_one_gpu,
+            "scaling_detail": scaling,
         }
         simt = load_json(os.path.join(ROOT, "profiles", "simt_efficiency.json"))
         if simt:
@@ -460,23 +521,46 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
         return statistics.median(ms) / reps
 
     c = I.C1
-    w = sr.divloop_workload(c.p_u32, c.fma_count, advance=c.advance_unroll)
     n_units = c.n_threads * c.iters
     exp_calls = None
     res = {}
-    # T = 16 is the config's threshold; T = 8 the best of the sweep with run-ahead lanes
-    # taking up to 8 iterations per round (tools/exp_dl_adv.sh); T = 32 = wait for every
-    # lane (Fig. 1(b))
-    for name, mode, thr in (("pdom", sr.PDOM, 0), ("spec_t16", sr.SPEC_LOOP, 16),
-                            ("spec_t8", sr.SPEC_LOOP, 8), ("spec_t32", sr.SPEC_LOOP, 32)):
+    # as written (one Philox draw per iteration, in program order) and with the
+    # conditions of 64 iterations evaluated together (prolog_batch, reading Q5') --
+    # both kernels get the same prolog.  V = run-ahead iterations per advance round
+    # (V = 1: the paper's one vote per iteration; V = 8 the default).  T = 16 is the
+    # config's threshold; T = 32 = wait for every lane (Fig. 1(b)).
+    runs = (("pdom", sr.PDOM, 0, 1, 0), ("spec_t16", sr.SPEC_LOOP, 16, c.advance_unroll, 0),
+            ("spec_t16_v1", sr.SPEC_LOOP, 16, 1, 0), ("spec_t8", sr.SPEC_LOOP, 8, c.advance_unroll, 0),
+            ("spec_t32", sr.SPEC_LOOP, 32, c.advance_unroll, 0),
+            ("pdom_batch", sr.PDOM, 0, 1, 64),
+            ("spec_t16_batch", sr.SPEC_LOOP, 16, c.advance_unroll, 64),
+            ("spec_t16_v1_batch", sr.SPEC_LOOP, 16, 1, 64),
+            ("spec_t8_batch", sr.SPEC_LOOP, 8, c.advance_unroll, 64),
+            ("spec_t32_batch", sr.SPEC_LOOP, 32, c.advance_unroll, 64))
+    for name, mode, thr, V, batch in runs:
+        w = sr.divloop_workload(c.p_u32, c.fma_count, advance=V, batch=batch)
         t = graph_time(w, c.n_threads, c.iters, mode, thr)
         sr.sr_run(w, c.n_threads, c.iters, I.PRIMARY_SEED, mode, thr)
         exp_calls = int(ctx.region(w, c.n_threads, sr.T_COUNTERS, torch.int64)[0].item())
         res[name] = {"value": n_units / (t * 1e-3), "unit": "thread-iterations/s", "ms": t,
+                     "advance_unroll": V, "prolog_batch": batch,
                      "fma_frac_of_peak": exp_calls * c.fma_count / (t * 1e-3) / fma_peak}
-    res["speedup_t16_vs_pdom"] = res["spec_t16"]["value"] / res["pdom"]["value"]
-    res["speedup_t8_vs_pdom"] = res["spec_t8"]["value"] / res["pdom"]["value"]
+    for k in ("t16", "t16_v1", "t8", "t32"):
+        res[f"speedup_{k}_vs_pdom"] = res[f"spec_{k}"]["value"] / res["pdom"]["value"]
+        res[f"speedup_{k}_batch_vs_pdom_batch"] = (res[f"spec_{k}_batch"]["value"] /
+                                                  res["pdom_batch"]["value"])
     res["expensive_calls"] = exp_calls
+    # issue roofline: useful work = the as-written PDOM kernel's thread-instructions
+    # (ncu, profiles/simt_efficiency.json), peak = 592 SMSPs x 32 lanes x f
+    simt = load_json(os.path.join(ROOT, "profiles", "simt_efficiency.json")) or {}
+    ti = (simt.get("divloop_pdom") or {}).get("thread_inst")
+    if ti:
+        peak = 592 * 32 * f_mhz * 1e6
+        res["issue_roofline"] = {
+            "thread_inst": ti,
+            "frac": {k: ti / (v["ms"] * 1e-3) / peak for k, v in res.items()
+                     if isinstance(v, dict) and "ms" in v},
+            "basis": "as-written PDOM thread-inst (ncu) / time / (592 x 32 x sm_max_mhz)"}
     out["divloop"] = res
 
     c = I.C2
@@ -491,10 +575,13 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
 
     # NEXT-1: RSBench-shaped nested trip-count loop (Fig. 3), PDOM vs Loop Merge
     c = I.NEXT1
-    w = sr.rsbench_workload(c.fma_count, unroll=c.merge_unroll)
     res = {}
-    for name, mode, thr in (("pdom", sr.PDOM, 0), (f"spec_t{c.threshold}", sr.SPEC_LOOP,
-                                                   c.threshold)):
+    # default: the warp task pool; "_static": lane l runs thread l's lookups itself
+    for name, mode, thr, flags in (("pdom", sr.PDOM, 0, 0),
+                                   (f"spec_t{c.threshold}", sr.SPEC_LOOP, c.threshold, 0),
+                                   (f"spec_t{c.threshold}_static", sr.SPEC_LOOP, c.threshold,
+                                    sr.F_STATIC)):
+        w = sr.rsbench_workload(c.fma_count, unroll=c.merge_unroll, flags=flags)
         t = graph_time(w, c.n_threads, c.iters, mode, thr, reps=5)
         sr.sr_run(w, c.n_threads, c.iters, I.PRIMARY_SEED, mode, thr)
         nucs = int(ctx.region(w, c.n_threads, sr.T_COUNTERS, torch.int64)[0].item())
@@ -508,10 +595,14 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
     # ... with an expensive task fetch (2048-FMA prolog, Fig. 9's XSBench case):
     # refilling idle lanes costs more, the best threshold drops (T = 32 shown too)
     c = I.NEXT1_FETCH
-    w = sr.rsbench_workload(c.fma_count, prolog_fma=c.prolog_fma, unroll=c.merge_unroll)
     res = {"prolog_fma": c.prolog_fma}
-    for name, mode, thr in (("pdom", sr.PDOM, 0), (f"spec_t{c.threshold}", sr.SPEC_LOOP,
-                                                   c.threshold), ("spec_t32", sr.SPEC_LOOP, 32)):
+    for name, mode, thr, flags in (("pdom", sr.PDOM, 0, 0),
+                                   (f"spec_t{c.threshold}", sr.SPEC_LOOP, c.threshold, 0),
+                                   ("spec_t32", sr.SPEC_LOOP, 32, 0),
+                                   (f"spec_t{c.threshold}_static", sr.SPEC_LOOP, c.threshold,
+                                    sr.F_STATIC)):
+        w = sr.rsbench_workload(c.fma_count, prolog_fma=c.prolog_fma, unroll=c.merge_unroll,
+                                flags=flags)
         t = graph_time(w, c.n_threads, c.iters, mode, thr, reps=5)
         res[name] = {"value": c.n_threads * c.iters / (t * 1e-3), "unit": "lookups/s", "ms": t}
     res["speedup_vs_pdom"] = res[f"spec_t{c.threshold}"]["value"] / res["pdom"]["value"]

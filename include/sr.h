@@ -64,7 +64,13 @@ typedef enum {
 #define SR_F_SCHED 1u   /* also write per-warp schedule counters (instrumented kernels) */
 #define SR_F_STATIC 2u  /* MCML / PATHTRACE: static task->lane assignment (lane l owns tasks
                            l + k*n_threads) instead of the default dynamic per-warp claiming.
-                           Results are identical; only the schedule differs. */
+                           RSBENCH + SR_SPEC_LOOP: lane l runs thread l's lookups itself
+                           instead of the default warp task pool (idle lanes claim the
+                           warp's next lookup in lane order; per-lookup xs staged in shared
+                           memory, (block/32)*(iters*32+32)*4 bytes per CTA, and summed per
+                           thread in program order at the end; above 160 KB the static
+                           assignment is used).  Results are identical; only the schedule
+                           differs. */
 #define SR_F_COARSE 4u  /* PATHTRACE + SR_SPEC_LOOP: merge at bounce granularity (one release =
                            traversal + shading of one bounce) instead of the default BVH-node
                            granularity (one release = one node visit). Results are identical. */
@@ -85,6 +91,14 @@ typedef struct {
   uint32_t advance_unroll; /* SR_SPEC_LOOP: iterations a run-ahead lane may take in
                           one advance round before it parks (0 = 1, reading Q5).
                           Results are identical for every value.               */
+  uint32_t prolog_batch; /* both modes: 0 or 1 = each iteration's Prolog (its one
+                          Philox draw, reading R3) evaluated in program order,
+                          one draw at a time, as Fig. 2(a) is written; 64 = a lane
+                          evaluates the divergent conditions of up to 64 of its
+                          iterations together (independent counters, ILP) into a
+                          64-bit mask, and redraws only the iterations that call
+                          Expensive() (reading Q5').  Other values: SR_E_INVALID.
+                          Results and schedule counters are identical.          */
 } sr_divloop_params;
 
 typedef struct {

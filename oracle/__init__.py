@@ -304,6 +304,19 @@ def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32, U=1):
     return o.as_dict(LM)
 
 
+def ws_loopmerge_pool(nsteps, T, U=1, W=32):
+    """Loop Merge over the warp's task pool: nsteps [n_valid, K] uint32 (task k of
+    thread l); task q = k * n_valid + l is claimed by idle lanes in lane order."""
+    nsteps = np.ascontiguousarray(nsteps, np.uint32)
+    n_valid, K = nsteps.shape
+    o = WsCounts()
+    L = lib()
+    L.ws_loopmerge_pool.argtypes = [C.POINTER(C.c_uint32), C.c_uint32, C.c_uint32, C.c_uint32,
+                                    C.c_uint32, C.c_uint32, C.POINTER(WsCounts)]
+    L.ws_loopmerge_pool(_p(nsteps, C.c_uint32), W, n_valid, K, T, U, C.byref(o))
+    return o.as_dict(LM)
+
+
 def ws_loopmerge_defer_raw(nsteps, ev_flat, ev_off, T, Tb, W=32):
     """Loop Merge + nested Iteration Delay of the boundary sub-step."""
     nsteps = np.ascontiguousarray(nsteps, np.uint32)

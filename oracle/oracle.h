@@ -184,6 +184,14 @@ void ws_commoncall(const uint8_t* arm, uint32_t W, uint32_t n_valid, int mode, w
 void ws_loopmerge_unrolled(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
                            uint32_t W, uint32_t n_valid, uint32_t K, int mode, uint32_t T,
                            uint32_t U, ws_counts* out);
+/* Loop Merge over a warp-shared task pool (Loop Merge's refill, with
+ * the n_valid*K tasks of the warp's threads as one queue): task q is task
+ * k = q / n_valid of thread q % n_valid (nsteps[l*K+k] as above); in an advance
+ * round every one of the W lanes that is not in a task is in R, and the first
+ * |R| unclaimed tasks go to R's lanes in lane order; the pool empty -> R = {}.
+ * U = steps per release as in ws_loopmerge_unrolled.  SPEC rule only. */
+void ws_loopmerge_pool(const uint32_t* nsteps, uint32_t W, uint32_t n_valid, uint32_t K,
+                       uint32_t T, uint32_t U, ws_counts* out);
 /* Loop Merge + nested Iteration Delay of the boundary sub-step (warpsim.c) */
 void ws_loopmerge_defer(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
                         uint32_t W, uint32_t n_valid, uint32_t K, uint32_t T, uint32_t Tb,

@@ -236,6 +236,52 @@ void ws_loopmerge_unrolled(const uint32_t* nsteps, const or_event* ev, const uin
   }
 }
 
+/* Loop Merge over a warp-shared pool of the warp's tasks (see oracle.h). */
+void ws_loopmerge_pool(const uint32_t* nsteps, uint32_t W, uint32_t n_valid, uint32_t K,
+                       uint32_t T, uint32_t U, ws_counts* o) {
+  if (U == 0) U = 1;
+  if (T == 0 || T > 32) T = 32;
+  if (W > 32) W = 32;
+  if (n_valid > W) n_valid = W;
+  memset(o, 0, sizeof *o);
+  const uint32_t valid = n_valid >= 32 ? 0xffffffffu : ((1u << n_valid) - 1u);
+  const uint32_t all = W >= 32 ? 0xffffffffu : ((1u << W) - 1u);
+  const uint64_t pool = (uint64_t)n_valid * K;
+  uint64_t qnext = 0;
+  uint32_t alive = 0, left[32] = {0};  /* steps left in the lane's task */
+  hit(o, WS_LM_ENTRY, valid);
+  for (;;) {
+    const uint32_t P = alive;
+    const uint32_t R = qnext < pool ? (all & ~alive) : 0u;
+    if (!P && !R) break;
+    o->rounds += 1;
+    hit(o, WS_LM_ROUND, all);
+    if ((uint32_t)__builtin_popcount(P) >= T || !R) {
+      hit(o, WS_LM_RELEASE, P);
+      uint32_t S = P;
+      for (uint32_t r = 0; r < U && S; ++r) {
+        hit(o, WS_LM_STEP, S);
+        for (uint32_t l = 0; l < W; ++l) {
+          if (!(S >> l & 1u)) continue;
+          if (--left[l] == 0) { alive &= ~(1u << l); S &= ~(1u << l); }
+        }
+      }
+    } else {
+      hit(o, WS_LM_ADVANCE, R);
+      uint32_t got = 0;
+      for (uint32_t l = 0; l < W; ++l) {   /* lane order */
+        if (!(R >> l & 1u) || qnext >= pool) continue;
+        const uint64_t q = qnext++;
+        const uint32_t owner = (uint32_t)(q % n_valid), k = (uint32_t)(q / n_valid);
+        left[l] = nsteps[(uint64_t)owner * K + k];
+        if (left[l]) alive |= 1u << l;
+        got |= 1u << l;
+      }
+      hit(o, WS_LM_LAUNCH, got);
+    }
+  }
+}
+
 /* ------------------------------------------------------------------ */
 /* Loop Merge with a second, nested prediction: Iteration Delay of the rare
  * boundary sub-step (two concurrent predictions).  A step is

@@ -14,8 +14,18 @@
 //            epilog and the next lookup's prolog while the others continue, as
 //            in Fig. 3(b)(iii); the inner body runs with the lanes that have
 //            nuclides left once popc >= T (or nobody can refill).
-// One lane = one thread of the problem (static); the lookup order and the
-// nuclide order of each lane are program order, so the float sums are
+// Task sources of rs_spec:
+//   static  (SR_F_STATIC) lane l of the warp is thread l of the problem and runs
+//           its lookups k = 0..iters-1 itself, in program order;
+//   pool    (default) the warp's 32 x iters lookups form one pool: an idle lane
+//           claims the next lookup q (lookup k = q / nv of thread q % nv, nv =
+//           valid threads of the warp) in lane order, so a lane whose lookups
+//           were light keeps working while the heavy 321-nuclide ones finish --
+//           no per-lane tail (the MC kernels' dynamic claiming, inside a warp).
+//           Each lookup's xs lands in shared memory at [k][thread]; at the end
+//           thread l sums its own xs in k order.
+// Either way every lookup's nuclide order is program order and each thread's
+// acc is the in-order sum of its lookups' xs, so the float results are
 // schedule-free (reading R8).
 #include <cmath>
 
@@ -26,6 +36,7 @@ namespace sr {
 namespace {
 
 constexpr uint32_t kMats = 12, kNuclides = 355;
+constexpr uint64_t kRsPoolSmemMax = 160 * 1024;  // pool smem per CTA; above it: static
 __constant__ uint32_t c_nucs[kMats] = {321, 5, 4, 4, 27, 21, 21, 21, 21, 21, 9, 9};
 
 struct RsArgs {
@@ -113,16 +124,28 @@ __global__ void __launch_bounds__(SR_RS_MAXT) rs_pdom(const RsArgs a) {
   finish(a, g, valid, acc, nucs, a.iters, r, rl, a.iters, a.iters * (uint32_t)__popc(__ballot_sync(kFull, valid)));
 }  // @sr-region END
 
-template <int ROUNDS, int PROLOG, bool SCHED>
+template <int ROUNDS, int PROLOG, bool SCHED, bool POOL>
 __global__ void __launch_bounds__(SR_RS_MAXT) rs_spec(const RsArgs a) {
+  extern __shared__ float rs_xs[];  // POOL: per warp xs[iters][32], then nucs[32]
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
   const bool valid = g < a.n;
-  const uint64_t t = a.t0 + g;
+  uint64_t t = a.t0 + g;
   float acc = 0.0f, xs = 0.0f, E = 0.0f;
   uint32_t nucs = 0, k = 0, i = 0, N = 0, m = 0;
   bool busy = false;                       // inside a lookup's inner loop
   uint32_t rounds = 0, rel = 0, rel_lanes = 0, adv = 0, adv_lanes = 0;
-  uint32_t E_mask = __ballot_sync(kFull, !valid || a.iters == 0);  // nothing left (Cancel)
+  // POOL state (warp-uniform): valid threads, pool size, next unclaimed lookup
+  const uint32_t nv = POOL ? (uint32_t)__popc(__ballot_sync(kFull, valid)) : 0u;
+  const uint32_t pool = nv * a.iters;
+  uint32_t qnext = 0, own = 0;             // own: thread (lane of the warp) of the lookup
+  float* const xw = rs_xs + (threadIdx.x >> 5) * (a.iters * 32u + 32u);
+  uint32_t* const nw = reinterpret_cast<uint32_t*>(xw + a.iters * 32u);
+  if constexpr (POOL) {
+    nw[lane_id()] = 0u;
+    __syncwarp();
+  }
+  uint32_t E_mask = POOL ? (pool == 0u ? kFull : 0u)                 // nothing left (Cancel)
+                         : __ballot_sync(kFull, !valid || a.iters == 0);
   uint32_t P = __ballot_sync(kFull, busy);  // round ballot, re-taken at the latch
   for (;;) {
     const uint32_t R = ~(P | E_mask);  // @sr-region ROUND:full
@@ -138,15 +161,32 @@ __global__ void __launch_bounds__(SR_RS_MAXT) rs_spec(const RsArgs a) {
           xs = xs + body<ROUNDS>(E, m, i, a.rounds);
           i = i + 1u;
           if (i == N) {                    // inner loop done: Epilog
-            acc = acc + xs;
-            nucs += N;
+            if constexpr (POOL) {
+              xw[(k - 1u) * 32u + own] = xs;  // k - 1: the lookup this lane holds
+              atomicAdd(&nw[own], N);
+            } else {
+              acc = acc + xs;
+              nucs += N;
+            }
             busy = false;
           }
         }
       }
     } else {
       if constexpr (SCHED) { ++adv; adv_lanes += __popc(R); }  // @sr-region ADVANCE:full
-      if ((R >> lane_id()) & 1u) {
+      bool go = (R >> lane_id()) & 1u;
+      if constexpr (POOL) {
+        // claim in lane order: lookup q = qnext + rank among the idle lanes
+        const uint32_t q = qnext + (uint32_t)__popc(R & lanemask_lt());
+        go = go && q < pool;
+        if (go) {
+          own = nv == 32u ? (q & 31u) : q % nv;
+          k = nv == 32u ? (q >> 5) : q / nv;
+          t = a.t0 + (g & ~31ull) + own;
+        }
+        qnext = min(pool, qnext + (uint32_t)__popc(R));
+      }
+      if (go) {
         const uint4 u = draw(k, kTagRs, t, a.keys);  // @sr-region LAUNCH
         m = pick(a, u.x);
         E = energy<PROLOG>(a, u.y);
@@ -156,22 +196,50 @@ __global__ void __launch_bounds__(SR_RS_MAXT) rs_spec(const RsArgs a) {
         busy = true;
         ++k;
       }
-      E_mask = __ballot_sync(kFull, !valid || k >= a.iters);  // @sr-region ADVANCE:full
+      if constexpr (POOL) E_mask = qnext >= pool ? kFull : 0u;  // @sr-region ADVANCE:full
+      else E_mask = __ballot_sync(kFull, !valid || k >= a.iters);
     }
     P = __ballot_sync(kFull, busy);  // @sr-region ROUND:full
+  }
+  if constexpr (POOL) {  // @sr-region ENTRY:full
+    __syncwarp();
+    if (valid) {  // this thread's lookups in program order
+      for (uint32_t kk = 0; kk < a.iters; ++kk) acc = acc + xw[kk * 32u + lane_id()];
+      nucs = nw[lane_id()];
+    }
   }
   finish(a, g, valid, acc, nucs, rounds, rel, rel_lanes, adv, adv_lanes);  // @sr-region ENTRY:full
 }  // @sr-region END
 
 template <bool SCHED>
-cudaError_t launch_t(const LaunchCtx& c, const RsArgs& a, int mode) {
+cudaError_t set_rs_smem(const RsArgs& a, int smem) {
+  cudaError_t e = cudaSuccess;
+  auto set = [&](auto kern) {
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  };
+  if (a.rounds == 8 && a.prolog_rounds == 0) set(rs_spec<8, 0, SCHED, true>);
+  else if (a.rounds == 8 && a.prolog_rounds == 256) set(rs_spec<8, 256, SCHED, true>);
+  else set(rs_spec<0, -1, SCHED, true>);
+  return e;
+}
+
+template <bool SCHED>
+cudaError_t launch_t(const LaunchCtx& c, const RsArgs& a, int mode, bool pool) {
   const uint32_t block = c.block;
   const uint64_t grid = (a.n + block - 1) / block;
   if (grid > 0x7fffffffull) return cudaErrorInvalidConfiguration;
-  record_launch((uint32_t)grid, block, 0);
   const bool spec = mode == SR_SPEC_LOOP;
-#define SR_RS(R, PR)                                                                \
-  (spec ? rs_spec<R, PR, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a)        \
+  // the pool's shared memory: per warp iters x 32 xs + 32 nuclide counts
+  const size_t smem = pool ? (size_t)(block / 32) * ((size_t)a.iters * 32 + 32) * 4 : 0;
+  record_launch((uint32_t)grid, block, (uint32_t)smem);
+  if (smem > 48 * 1024) {
+    cudaError_t e = set_rs_smem<SCHED>(a, (int)smem);
+    if (e != cudaSuccess) return e;
+  }
+#define SR_RS(R, PR)                                                                      \
+  (spec ? (pool ? rs_spec<R, PR, SCHED, true><<<(unsigned)grid, block, smem, c.stream>>>(a) \
+                : rs_spec<R, PR, SCHED, false><<<(unsigned)grid, block, 0, c.stream>>>(a)) \
         : rs_pdom<R, PR, SCHED><<<(unsigned)grid, block, 0, c.stream>>>(a))
   // compile-time shapes of the measured configurations (straight-line code,
   // static SASS costs for the simulator); anything else runs the generic one
@@ -183,6 +251,10 @@ cudaError_t launch_t(const LaunchCtx& c, const RsArgs& a, int mode) {
 }
 
 }  // namespace
+
+bool rs_pool_fits(uint32_t iters, uint32_t block) {
+  return (uint64_t)(block / 32) * ((uint64_t)iters * 32 + 32) * 4 <= kRsPoolSmemMax;
+}
 
 cudaError_t launch_rsbench(const LaunchCtx& c, const sr_workload& w, uint64_t n, uint32_t iters,
                            uint64_t seed, int mode, uint32_t T) {
@@ -207,7 +279,10 @@ cudaError_t launch_rsbench(const LaunchCtx& c, const sr_workload& w, uint64_t n,
   a.counters = reinterpret_cast<unsigned long long*>(c.ws + c.lay.off[SR_T_COUNTERS]);
   a.sched = (w.flags & SR_F_SCHED) ? reinterpret_cast<uint32_t*>(c.ws + c.lay.off[SR_T_SCHED])
                                    : nullptr;
-  return a.sched ? launch_t<true>(c, a, mode) : launch_t<false>(c, a, mode);
+  // the warp pool unless SR_F_STATIC, or its shared memory would not fit
+  const uint32_t block = c.block;
+  const bool pool = !(w.flags & SR_F_STATIC) && rs_pool_fits(iters, block);
+  return a.sched ? launch_t<true>(c, a, mode, pool) : launch_t<false>(c, a, mode, pool);
 }
 
 }  // namespace sr

@@ -95,6 +95,8 @@ MISMATCHED_ABSORBER = MCML(layers=((1.4, 5.0, 0.0, 0.0, 0.1),), nz=100, dz=0.001
 C1 = DivLoop()
 C2 = CommonCall()
 C3 = MCML()
+# configs[4]: 10^9 photons of C3 in total, sharded over 1/2/4/8 GPUs (strong scaling)
+C5_TOTAL_PHOTONS = 10**9
 
 
 # ---------------------------------------------------------------- config 4 scene

@@ -45,7 +45,8 @@ class Layer(C.Structure):
 
 
 class DivloopParams(C.Structure):
-    _fields_ = [("p_u32", C.c_uint32), ("fma_count", C.c_uint32), ("advance_unroll", C.c_uint32)]
+    _fields_ = [("p_u32", C.c_uint32), ("fma_count", C.c_uint32), ("advance_unroll", C.c_uint32),
+                ("prolog_batch", C.c_uint32)]
 
 
 class CommoncallParams(C.Structure):
@@ -207,9 +208,9 @@ def scene_image_host(tris, mat, mats, cam):
 
 # ------------------------------------------------------------------ workload builders
 def divloop_workload(p_u32=1 << 29, fma_count=1000, task_offset=0, flags=0, block=0,
-                     advance=0) -> Workload:
+                     advance=0, batch=0) -> Workload:
     w = Workload(kind=WL_DIVLOOP, flags=flags, task_offset=task_offset, block_threads=block)
-    w.divloop = DivloopParams(p_u32, fma_count, advance)
+    w.divloop = DivloopParams(p_u32, fma_count, advance, batch)
     return w
 
 

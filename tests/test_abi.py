@@ -93,6 +93,11 @@ def test_run_validation_before_state():
     bad = sr.divloop_workload(block=48)
     with pytest.raises(sr.SRError):
         sr.sr_run(bad, 64, 1, 1, sr.PDOM, 0)
+    for batch in (2, 8, 63, 65):
+        bad = sr.divloop_workload(batch=batch)
+        with pytest.raises(sr.SRError) as e:
+            sr.sr_run(bad, 64, 1, 1, sr.PDOM, 0)
+        assert e.value.code == sr.SR_E_INVALID and "prolog_batch" in str(e.value)
 
 
 def test_mcml_param_validation():

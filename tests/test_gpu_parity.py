@@ -256,6 +256,61 @@ def test_divloop_schedule_matches_simulator(ctx, mode, T):
             assert (g[3], g[4]) == s["ADVANCE"] and s["PROLOG"] == s["ADVANCE"], wi
 
 
+# batched prolog (prolog_batch = 64, reading Q5'): same bits, same schedule
+@pytest.mark.parametrize("mode,T,V", [(sr.PDOM, 0, 1), (sr.SPEC_LOOP, 1, 1), (sr.SPEC_LOOP, 16, 1),
+                                      (sr.SPEC_LOOP, 16, 8), (sr.SPEC_LOOP, 32, 8),
+                                      (sr.SPEC_LOOP, 8, 100)])
+@pytest.mark.parametrize("n,iters,off", [(1000, 64, 0), (333, 200, 0), (65, 63, 0),
+                                         (100, 0, 0), (1, 129, 0), (97, 65, (1 << 40) + 7)])
+def test_divloop_batch_bit_exact(ctx, mode, T, V, n, iters, off):
+    """iters > 64 crosses mask windows (200 = 3 x 64 + 8; 129; 65), V = 100 spans them"""
+    acc_o, cnt_o = oracle.divloop(off, n, iters, 7)
+    w = sr.divloop_workload(task_offset=off, block=64, advance=V, batch=64)
+    acc, cnt, tot = run_divloop(ctx, w, n, iters, 7, mode, T)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(cnt, cnt_o)
+    assert tot[0] == cnt_o.sum()
+
+
+@pytest.mark.parametrize("kw", [dict(p_u32=0), dict(p_u32=0xFFFFFFFF), dict(fma_count=8)])
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 16)])
+def test_divloop_batch_edge_cases(ctx, kw, mode, T):
+    p = dict(p_u32=1 << 29, fma_count=1000); p.update(kw)
+    acc_o, cnt_o = oracle.divloop(0, 100, 70, 7, p["p_u32"], p["fma_count"])
+    acc, cnt, _ = run_divloop(ctx, sr.divloop_workload(batch=64, advance=8, **kw), 100, 70, 7,
+                              mode, T)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(cnt, cnt_o)
+
+
+def test_divloop_batch_full_config(ctx):
+    c = I.C1
+    acc_o, cnt_o = oracle.divloop(0, c.n_threads, c.iters, I.PRIMARY_SEED, c.p_u32, c.fma_count)
+    for mode, T in ((sr.PDOM, 0), (sr.SPEC_LOOP, 16), (sr.SPEC_LOOP, 1)):
+        w = sr.divloop_workload(c.p_u32, c.fma_count, advance=c.advance_unroll, batch=64)
+        acc, cnt, _ = run_divloop(ctx, w, c.n_threads, c.iters, I.PRIMARY_SEED, mode, T)
+        assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32)), (mode, T)
+        assert np.array_equal(cnt, cnt_o), (mode, T)
+
+
+@pytest.mark.parametrize("mode,T,V", [(sr.PDOM, 0, 1), (sr.SPEC_LOOP, 16, 1), (sr.SPEC_LOOP, 16, 8),
+                                      (sr.SPEC_LOOP, 4, 3)])
+def test_divloop_batch_schedule_matches_simulator(ctx, mode, T, V):
+    n, iters = 2000, 64
+    w = sr.divloop_workload(flags=sr.F_SCHED, block=64, advance=V, batch=64)
+    run_divloop(ctx, w, n, iters, I.PRIMARY_SEED, mode, T)
+    sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    want = oracle.divloop_wants(0, n, iters, I.PRIMARY_SEED)
+    for wi in range((n + 31) // 32):
+        s = oracle.ws_divloop(want[32 * wi:32 * wi + 32],
+                              oracle.PDOM if mode == sr.PDOM else oracle.SPEC_LOOP, T,
+                              V=V if mode == sr.SPEC_LOOP else 1)
+        g = sched[wi]
+        assert (g[1], g[2]) == s["EXPENSIVE"], wi
+        if mode == sr.SPEC_LOOP:
+            assert g[0] == s["rounds"] and (g[3], g[4]) == s["ADVANCE"], wi
+
+
 # ------------------------------------------------------------------ config 2
 def run_cc(ctx, w, n, iters, seed, mode):
     ctx.ensure(sr.sr_workspace_bytes(w, n))

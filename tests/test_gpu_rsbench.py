@@ -35,10 +35,11 @@ def run(ctx, w, n, iters, seed, mode, T):
 @pytest.mark.parametrize("seed", I.SEEDS)
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 4),
                                     (sr.SPEC_LOOP, 16), (sr.SPEC_LOOP, 32)])
-def test_rsbench_bit_exact_small(ctx, seed, mode, T):
+@pytest.mark.parametrize("flags", [0, sr.F_STATIC])   # warp task pool (default) / static
+def test_rsbench_bit_exact_small(ctx, seed, mode, T, flags):
     n, iters = 700, 6
     acc_o, nuc_o = oracle.rsbench(0, n, iters, seed)
-    acc, nuc, cnt = run(ctx, sr.rsbench_workload(block=64), n, iters, seed, mode, T)
+    acc, nuc, cnt = run(ctx, sr.rsbench_workload(block=64, flags=flags), n, iters, seed, mode, T)
     assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
     assert np.array_equal(nuc, nuc_o)
     assert cnt[0] == nuc_o.sum()
@@ -58,7 +59,7 @@ def test_rsbench_unrolled_merge_bit_exact(ctx, T, U):
 @pytest.mark.parametrize("T,U", [(24, 2), (32, 4)])
 def test_rsbench_unrolled_schedule_matches_simulator(ctx, T, U):
     n, iters = 256, 8
-    w = sr.rsbench_workload(flags=sr.F_SCHED, block=64, unroll=U)
+    w = sr.rsbench_workload(flags=sr.F_SCHED | sr.F_STATIC, block=64, unroll=U)
     run(ctx, w, n, iters, 5, sr.SPEC_LOOP, T)
     sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
     _, _, trips = oracle.rsbench(0, n, iters, 5, fma_count=0, trips=True)
@@ -72,7 +73,7 @@ def test_rsbench_unrolled_schedule_matches_simulator(ctx, T, U):
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 4), (sr.SPEC_LOOP, 32)])
 def test_rsbench_schedule_matches_simulator(ctx, mode, T):
     n, iters = 256, 8
-    w = sr.rsbench_workload(flags=sr.F_SCHED, block=64)
+    w = sr.rsbench_workload(flags=sr.F_SCHED | sr.F_STATIC, block=64)
     run(ctx, w, n, iters, 5, mode, T)
     sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
     _, _, trips = oracle.rsbench(0, n, iters, 5, fma_count=0, trips=True)
@@ -83,6 +84,34 @@ def test_rsbench_schedule_matches_simulator(ctx, mode, T):
         assert (g[1], g[2]) == s["STEP"], wi
         if mode == sr.SPEC_LOOP:
             assert g[0] == s["rounds"] and (g[3], g[4]) == s["LAUNCH"], wi
+
+
+@pytest.mark.parametrize("n,iters,T,U,block", [(700, 6, 24, 12, 64), (333, 5, 4, 1, 96),
+                                               (31, 40, 32, 3, 256), (1, 7, 16, 2, 32),
+                                               (100, 0, 24, 12, 64), (65, 129, 24, 12, 128)])
+def test_rsbench_pool_bit_exact(ctx, n, iters, T, U, block):
+    """the warp task pool: ragged warps (a partial warp's idle lanes work on its
+    threads' lookups), one thread, zero lookups, many lookups per thread"""
+    acc_o, nuc_o = oracle.rsbench(11, n, iters, 3)
+    w = sr.rsbench_workload(block=block, task_offset=11, unroll=U)
+    acc, nuc, cnt = run(ctx, w, n, iters, 3, sr.SPEC_LOOP, T)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(nuc, nuc_o)
+    assert cnt[0] == nuc_o.sum()
+
+
+@pytest.mark.parametrize("T,U,n", [(24, 1, 256), (24, 12, 256), (4, 3, 200), (32, 2, 77)])
+def test_rsbench_pool_schedule_matches_simulator(ctx, T, U, n):
+    iters = 8
+    w = sr.rsbench_workload(flags=sr.F_SCHED, block=64, unroll=U)
+    run(ctx, w, n, iters, 5, sr.SPEC_LOOP, T)
+    sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    _, _, trips = oracle.rsbench(0, n, iters, 5, fma_count=0, trips=True)
+    for wi in range((n + 31) // 32):
+        s = oracle.ws_loopmerge_pool(trips[32 * wi:32 * wi + 32], T, U=U)
+        g = sched[wi]
+        assert g[0] == s["rounds"] and (g[1], g[2]) == s["RELEASE"], wi
+        assert (g[3], g[4]) == s["ADVANCE"], wi
 
 
 def test_rsbench_full_config_sampled(ctx):

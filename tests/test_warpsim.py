@@ -184,3 +184,56 @@ def test_divloop_advance_unroll_invariants():
             if T == 32:
                 assert s["EXPENSIVE"] == base["EXPENSIVE"]
             assert s["rounds"] <= oracle.ws_divloop(want, oracle.SPEC_LOOP, T)["rounds"]
+
+
+# ------------------------------------------------------------------ task pool
+def _pool_makespan(ns, W):
+    """Greedy list schedule of the pool (task q = k*n_valid + l, in order) on W
+    unit-speed lanes, ties to the lower lane: written independently of the
+    simulator, as an event simulation over time."""
+    n_valid, K = ns.shape
+    tasks = [int(ns[q % n_valid, q // n_valid]) for q in range(n_valid * K)]
+    free_at = [0] * W
+    end = 0
+    for d in tasks:
+        t = min(free_at)
+        lane = free_at.index(t)   # lowest lane among the earliest free
+        free_at[lane] = t + d
+        end = max(end, t + d)
+    return end
+
+
+@pytest.mark.parametrize("K,vals", [(1, [1, 2, 3, 4]), (2, [1, 2, 3]), (3, [1, 3])])
+def test_pool_bruteforce_4_lanes(K, vals):
+    """every trip-count combination in {1,2,3}^(4K) of a 4-lane warp:
+    conservation, T = 1 runs the pool batch by batch (STEP executions = sum of
+    each batch's longest task), T = W is greedy list scheduling (STEP executions
+    = its makespan), U > 1 never adds rounds or releases"""
+    W = 4
+    for combo in itertools.product(vals, repeat=W * K):
+        ns = np.array(combo, np.uint32).reshape(W, K)
+        tot = int(ns.sum())
+        s1 = oracle.ws_loopmerge_pool(ns, 1, W=W)
+        sW = oracle.ws_loopmerge_pool(ns, W, W=W)
+        for s in (s1, sW):
+            assert s["STEP"][1] == tot and s["RELEASE"] == s["STEP"]
+            assert s["LAUNCH"][1] == W * K
+            assert s["rounds"] == s["RELEASE"][0] + s["ADVANCE"][0]
+        tasks = [int(ns[q % W, q // W]) for q in range(W * K)]
+        assert s1["STEP"][0] == sum(max(tasks[b:b + W]) for b in range(0, W * K, W))
+        assert s1["ADVANCE"][0] == K
+        assert sW["STEP"][0] == _pool_makespan(ns, W)
+        for U in (2, 3):
+            su = oracle.ws_loopmerge_pool(ns, W, U=U, W=W)
+            assert su["STEP"][1] == tot and su["LAUNCH"][1] == W * K
+            assert su["RELEASE"][0] <= sW["RELEASE"][0] and su["rounds"] <= sW["rounds"]
+
+
+def test_pool_partial_warp_and_hand_schedule():
+    # 3 valid threads x 2 tasks on a 4-lane warp: the 4th lane works too
+    ns = np.array([[3, 1], [2, 2], [1, 5]], np.uint32)
+    s = oracle.ws_loopmerge_pool(ns, 4, W=4)
+    # tasks q0..q5 = 3,2,1,1,2,5; lanes 0..3 take q0..q3 at t=0 (3,2,1,1);
+    # t=1: lanes 2,3 free -> q4 (2) on lane 2, q5 (5) on lane 3 -> ends at 6
+    assert s["STEP"] == (6, 14) and s["LAUNCH"] == (2, 6) and s["ENTRY"] == (1, 3)
+    assert s["ADVANCE"] == (2, 4 + 2)   # round 1: all 4 lanes idle; t=1: lanes 2, 3

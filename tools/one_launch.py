@@ -24,13 +24,15 @@ ap.add_argument("--iters", type=int, default=0, help="MCML photons per lane (def
 ap.add_argument("--unroll", type=int, default=I.C3.merge_unroll,
                 help="MCML merge unroll (default: the bench's, configs[2])")
 ap.add_argument("--pt-flags", type=int, default=0, help="extra PATHTRACE flags (F_NOSPLIT = 8)")
+ap.add_argument("--dl-batch", type=int, default=0, help="divloop prolog_batch (0 or 64)")
+ap.add_argument("--rs-flags", type=int, default=0, help="extra RSBENCH flags (F_STATIC = 2)")
 a = ap.parse_args()
 modes = a.modes.split(",")
 ctx = sr.Context.create(0, 1 << 20)
 seed = I.PRIMARY_SEED
 if "divloop" in a.what:
     c = I.C1
-    w = sr.divloop_workload(c.p_u32, c.fma_count, advance=c.advance_unroll)
+    w = sr.divloop_workload(c.p_u32, c.fma_count, advance=c.advance_unroll, batch=a.dl_batch)
     ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
     for md in modes:
         sr.sr_run(w, c.n_threads, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
@@ -53,7 +55,7 @@ if "mcml" in a.what:
                   0 if md == "pdom" else a.threshold)
 if "rsbench" in a.what:
     c = I.NEXT1
-    w = sr.rsbench_workload(c.fma_count, unroll=c.merge_unroll)
+    w = sr.rsbench_workload(c.fma_count, unroll=c.merge_unroll, flags=a.rs_flags)
     ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
     for md in modes:
         sr.sr_run(w, c.n_threads, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
