@@ -81,6 +81,11 @@ typedef enum {
                            larger waiting group (soft barrier T) while the other lanes wait.
                            Results and counters are identical (each lane's traversal order is
                            the same). */
+#define SR_F_MATGROUP 16u /* PATHTRACE + SR_SPEC_LOOP, split node merge (the default): NEXT-3's
+                           same-material grouping of the shading step -- in an
+                           advance round the lanes that must shade a hit are grouped by material
+                           kind (__match_any_sync); only the largest group shades, the others
+                           wait for a later advance round.  Results and counters are identical. */
 
 #define SR_MAX_LAYERS 8
 typedef struct { float n, mua, mus, g, d; } sr_layer;  /* -, 1/cm, 1/cm, -, cm */

@@ -31,7 +31,7 @@ DL = dict(ENTRY=0, PROLOG=1, EXPENSIVE=2, EPILOG=3, ROUND=4, RELEASE=5, ADVANCE=
 CC = dict(ENTRY=0, THEN=1, ELSE_PRE=2, CALL=3, ELSE_POST=4, MERGE=5)
 LM = dict(ENTRY=0, LAUNCH=1, STEP=2, STEP_BOUNDARY=3, STEP_INTERACT=4, ROUND=5, RELEASE=6,
           ADVANCE=7, **{f"EV{b}": 8 + b for b in range(16)}, **{f"NEV{b}": 24 + b for b in range(16)},
-          A_RR=40, B_RR=41, B_REL=42, BI=43, A_TAIL=44)
+          A_RR=40, B_RR=41, B_REL=42, BI=43, A_TAIL=44, CLAIM=45, CLAIMIT=46, CHUNK=47)
 # MC step event bits (oracle.h OR_EV_*)
 EV_BOUNDARY, EV_SLEFT, EV_REFLECT, EV_EXIT, EV_TRANSMIT, EV_ROULETTE, EV_SPIN_AXIS, \
     EV_SPIN_GENERAL, EV_EXTERNAL, EV_MATCHED = 1, 2, 4, 8, 16, 32, 64, 128, 256, 512
@@ -301,6 +301,23 @@ def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32, U=1):
                             None if ev_flat is None else _p(ev_flat, C.c_uint16),
                             None if ev_off is None else _p(ev_off, C.c_uint64),
                             W, n_valid, K, mode, T, U, C.byref(o))
+    return o.as_dict(LM)
+
+
+def ws_loopmerge_stream(nsteps, mode, T, U=1, W=32, ev=None, ev_off=None):
+    """Loop Merge / PDOM with dynamic claiming from one task stream (the MC
+    kernels' default task source): nsteps [Q] uint32, optional events."""
+    nsteps = np.ascontiguousarray(nsteps, np.uint32)
+    o = WsCounts()
+    L = lib()
+    L.ws_loopmerge_stream.argtypes = [C.POINTER(C.c_uint32), C.POINTER(C.c_uint16),
+                                      C.POINTER(C.c_uint64), C.c_uint32, C.c_uint64, C.c_int,
+                                      C.c_uint32, C.c_uint32, C.POINTER(WsCounts)]
+    if ev_off is not None:
+        ev_off = np.ascontiguousarray(ev_off, np.uint64)
+    L.ws_loopmerge_stream(_p(nsteps, C.c_uint32), None if ev is None else _p(ev, C.c_uint16),
+                          None if ev_off is None else _p(ev_off, C.c_uint64), W,
+                          nsteps.shape[0], mode, T, U, C.byref(o))
     return o.as_dict(LM)
 
 

@@ -162,6 +162,9 @@ enum { WS_LM_ENTRY = 0, WS_LM_LAUNCH, WS_LM_STEP, WS_LM_STEP_BOUNDARY,
                               lanes = parked set                                      */
        WS_LM_BI = 43,      /* matched boundary finished inside part A (no part B)     */
        WS_LM_A_TAIL = 44,  /* end of part A: interaction + matched-boundary lanes     */
+       WS_LM_CLAIM = 45,   /* dynamic claim: slow path entered (reservoir short)      */
+       WS_LM_CLAIMIT = 46, /* dynamic claim: slow-path loop iterations                */
+       WS_LM_CHUNK = 47,   /* dynamic claim: chunk fetches from the global counter   */
        WS_LM_NREG = 45 };
 #define WS_MAX_REG 48
 typedef struct {
@@ -192,6 +195,15 @@ void ws_loopmerge_unrolled(const uint32_t* nsteps, const or_event* ev, const uin
  * U = steps per release as in ws_loopmerge_unrolled.  SPEC rule only. */
 void ws_loopmerge_pool(const uint32_t* nsteps, uint32_t W, uint32_t n_valid, uint32_t K,
                        uint32_t T, uint32_t U, ws_counts* out);
+/* Loop Merge with the MC kernels' dynamic task claiming: the warp's W lanes
+ * take tasks q = 0..Q-1 of one stream (nsteps[q] steps, events at ev_off[q]) in
+ * claim order.  PDOM: each outer trip every lane claims one task (lane order);
+ * the loop ends when no lane got one.  SPEC: an advance round hands the next
+ * tasks to the idle lanes of R in lane order; a lane left without one is
+ * exhausted (E) from then on.  U = steps per release. */
+void ws_loopmerge_stream(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
+                         uint32_t W, uint64_t Q, int mode, uint32_t T, uint32_t U,
+                         ws_counts* out);
 /* Loop Merge + nested Iteration Delay of the boundary sub-step (warpsim.c) */
 void ws_loopmerge_defer(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
                         uint32_t W, uint32_t n_valid, uint32_t K, uint32_t T, uint32_t Tb,

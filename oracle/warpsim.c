@@ -236,6 +236,115 @@ void ws_loopmerge_unrolled(const uint32_t* nsteps, const or_event* ev, const uin
   }
 }
 
+/* Loop Merge over one stream of tasks claimed dynamically (see oracle.h).
+ * step_split is called with K = 0 and kk[l] = the lane's task index q.
+ * The claim itself is modelled as the kernels run it: a warp-level reservoir
+ * [rv_next, rv_end) refilled CHUNK tasks at a time from the stream; a claim
+ * for `need` lanes takes the fast path when the reservoir covers them, else a
+ * loop that fetches chunks (CHUNK) and serves lanes in lane order (CLAIMIT),
+ * stopping when the stream is empty. */
+#define WS_CHUNK 32u
+typedef struct { uint64_t next, end, fetch, Q; } ws_reservoir;
+
+/* serve `want` lanes in lane order; returns the mask served (tasks in kk[]) */
+static uint32_t ws_claim(ws_counts* o, ws_reservoir* rv, uint32_t want, uint32_t all,
+                         uint32_t* kk) {
+  const uint32_t need = (uint32_t)__builtin_popcount(want);
+  uint32_t served = 0, got = 0;
+  if (rv->end - rv->next < need) {
+    hit(o, WS_LM_CLAIM, all);
+    while (served < need) {
+      hit(o, WS_LM_CLAIMIT, all);
+      if (rv->next >= rv->end) {
+        hit(o, WS_LM_CHUNK, all);
+        if (rv->fetch >= rv->Q) break;
+        rv->next = rv->fetch;
+        rv->end = rv->fetch + WS_CHUNK < rv->Q ? rv->fetch + WS_CHUNK : rv->Q;
+        rv->fetch += WS_CHUNK;
+      }
+      const uint64_t avail = rv->end - rv->next;
+      const uint32_t take = (uint32_t)(avail < need - served ? avail : need - served);
+      served += take;
+      rv->next += take;
+    }
+  } else {
+    served = need;
+    rv->next += need;
+  }
+  /* the first `served` lanes of `want` (lane order) get consecutive tasks */
+  uint64_t q = rv->next - served;
+  uint32_t k = 0;
+  for (uint32_t l = 0; l < 32 && k < served; ++l) {
+    if (!(want >> l & 1u)) continue;
+    kk[l] = (uint32_t)q++;
+    got |= 1u << l;
+    ++k;
+  }
+  return got;
+}
+
+void ws_loopmerge_stream(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev_off,
+                         uint32_t W, uint64_t Q, int mode, uint32_t T, uint32_t U,
+                         ws_counts* o) {
+  if (U == 0) U = 1;
+  if (W > 32) W = 32;
+  memset(o, 0, sizeof *o);
+  const uint32_t all = W >= 32 ? 0xffffffffu : ((1u << W) - 1u);
+  uint32_t kk[32] = {0}, jj[32] = {0};
+  ws_reservoir rv = {0, 0, 0, Q};
+  hit(o, WS_LM_ENTRY, all);
+  if (mode == WS_PDOM) {
+    for (;;) {
+      const uint32_t H = ws_claim(o, &rv, all, all, kk);
+      if (!H) break;
+      for (uint32_t l = 0; l < W; ++l) jj[l] = 0;
+      hit(o, WS_LM_LAUNCH, H);
+      for (;;) {
+        uint32_t m = 0;
+        for (uint32_t l = 0; l < W; ++l)
+          if ((H >> l & 1u) && jj[l] < nsteps[kk[l]]) m |= 1u << l;
+        if (!m) break;
+        hit(o, WS_LM_STEP, m);
+        if (ev) step_split(o, ev, ev_off, 0, kk, jj, m);
+        for (uint32_t l = 0; l < W; ++l)
+          if (m >> l & 1u) jj[l] += 1;
+      }
+    }
+    return;
+  }
+  if (T == 0 || T > 32) T = 32;
+  uint32_t alive = 0, exhausted = 0;
+  for (;;) {
+    const uint32_t P = alive, R = all & ~alive & ~exhausted;
+    if (!P && !R) break;
+    o->rounds += 1;
+    hit(o, WS_LM_ROUND, all);
+    if ((uint32_t)__builtin_popcount(P) >= T || !R) {
+      hit(o, WS_LM_RELEASE, P);
+      uint32_t S = P;
+      for (uint32_t r = 0; r < U && S; ++r) {
+        hit(o, WS_LM_STEP, S);
+        if (ev) step_split(o, ev, ev_off, 0, kk, jj, S);
+        for (uint32_t l = 0; l < W; ++l) {
+          if (!(S >> l & 1u)) continue;
+          jj[l] += 1;
+          if (jj[l] >= nsteps[kk[l]]) { alive &= ~(1u << l); S &= ~(1u << l); }
+        }
+      }
+    } else {
+      hit(o, WS_LM_ADVANCE, R);
+      const uint32_t got = ws_claim(o, &rv, R, all, kk);
+      exhausted |= R & ~got;
+      for (uint32_t l = 0; l < W; ++l) {
+        if (!(got >> l & 1u)) continue;
+        jj[l] = 0;
+        if (nsteps[kk[l]]) alive |= 1u << l;
+      }
+      hit(o, WS_LM_LAUNCH, got);
+    }
+  }
+}
+
 /* Loop Merge over a warp-shared pool of the warp's tasks (see oracle.h). */
 void ws_loopmerge_pool(const uint32_t* nsteps, uint32_t W, uint32_t n_valid, uint32_t K,
                        uint32_t T, uint32_t U, ws_counts* o) {

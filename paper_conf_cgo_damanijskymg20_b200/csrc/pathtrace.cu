@@ -482,7 +482,12 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_PDOM) pt_pdom(const PtA
 // nesting level deeper (P:1514-1528 leaves nesting open), where the trip
 // count (nodes per ray) varies most.  SPLIT (with NODE): the node visit's
 // leaf triangle tests become their own region (trav_node / trav_leaf).
-template <bool SCHED, bool NODE, bool SPLIT = false>
+// MATG (with SPLIT, SR_F_MATGROUP): NEXT-3's same-material grouping
+// of the shading step -- the lanes of R that must shade a hit
+// are grouped by material kind with __match_any_sync; the largest group shades
+// in this advance round (ties: the group of the lowest lane), the others wait
+// in R for a later one.  A miss forms its own group.
+template <bool SCHED, bool NODE, bool SPLIT = false, bool MATG = false>
 __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) {
   const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -530,7 +535,20 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
         continue;
       }
       if constexpr (SCHED) { ++adv; adv_lanes += __popc(R); }
-      if ((R >> lane_id()) & 1u) {
+      bool go = (R >> lane_id()) & 1u;
+      if constexpr (MATG) {
+        const bool needs = go && p.alive;   // a finished traversal whose hit must be shaded
+        if (__ballot_sync(kFull, needs) != 0u) {
+          const uint32_t key = !needs ? 0xFFFFFFFFu
+                             : (tr.ib < 0 ? 4u : (uint32_t)__ldg(&a.mats[tr.mb].kind));
+          const uint32_t grp = __match_any_sync(kFull, key);
+          // largest group, ties to the lowest lane: maximise (size << 5) | (31 - lowest lane)
+          const uint32_t score = needs ? ((uint32_t)__popc(grp) << 5) | (31u - (__ffs(grp) - 1u)) : 0u;
+          const uint32_t best = __reduce_max_sync(kFull, score);
+          go = go && (!needs || score == best);
+        }
+      }
+      if (go) {
         if (p.alive) shade(a, p, tr);
         if (!p.alive && next_s < a.spp) {
           p.s = next_s++;
@@ -714,10 +732,15 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
     cudaFuncSetAttribute(pt_spec<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaFuncSetAttribute(pt_spec<false, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaFuncSetAttribute(pt_spec<true, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<false, true, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<true, true, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   }
   if (!spec) {
     if (a.sched) pt_pdom<true><<<gr, block, smem, c.stream>>>(a);
     else pt_pdom<false><<<gr, block, smem, c.stream>>>(a);
+  } else if (node && !(w.flags & SR_F_NOSPLIT) && (w.flags & SR_F_MATGROUP)) {
+    if (a.sched) pt_spec<true, true, true, true><<<gr, block, smem, c.stream>>>(a);
+    else pt_spec<false, true, true, true><<<gr, block, smem, c.stream>>>(a);
   } else if (node && !(w.flags & SR_F_NOSPLIT)) {
     if (a.sched) pt_spec<true, true, true><<<gr, block, smem, c.stream>>>(a);
     else pt_spec<false, true, true><<<gr, block, smem, c.stream>>>(a);

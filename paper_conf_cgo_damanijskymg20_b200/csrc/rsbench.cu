@@ -204,8 +204,8 @@ __global__ void __launch_bounds__(SR_RS_MAXT) rs_spec(const RsArgs a) {
   if constexpr (POOL) {  // @sr-region ENTRY:full
     __syncwarp();
     if (valid) {  // this thread's lookups in program order
-      for (uint32_t kk = 0; kk < a.iters; ++kk) acc = acc + xw[kk * 32u + lane_id()];
-      nucs = nw[lane_id()];
+      for (uint32_t kk = 0; kk < a.iters; ++kk) acc = acc + xw[kk * 32u + lane_id()];  // @sr-region PERK:full
+      nucs = nw[lane_id()];  // @sr-region ENTRY:full
     }
   }
   finish(a, g, valid, acc, nucs, rounds, rel, rel_lanes, adv, adv_lanes);  // @sr-region ENTRY:full

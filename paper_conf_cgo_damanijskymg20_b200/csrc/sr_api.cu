@@ -64,7 +64,8 @@ std::string check_workload(const sr_workload* w, uint64_t n_threads) {
   if (w->block_threads > max_block(w->kind))
     return "block_threads exceeds this workload's kernels' launch bound (" +
            std::to_string(max_block(w->kind)) + ")";
-  if (w->flags & ~(SR_F_SCHED | SR_F_STATIC | SR_F_COARSE | SR_F_NOSPLIT)) return "unknown flags";
+  if (w->flags & ~(SR_F_SCHED | SR_F_STATIC | SR_F_COARSE | SR_F_NOSPLIT | SR_F_MATGROUP))
+    return "unknown flags";
   switch (w->kind) {
     case SR_WL_DIVLOOP:
       if (w->divloop.fma_count % 8 != 0) return "divloop.fma_count must be a multiple of 8";

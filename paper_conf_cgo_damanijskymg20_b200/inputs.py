@@ -41,7 +41,8 @@ class RSBench:
     n_threads: int = 131072
     iters: int = 32             # lookups per thread (thread coarsening)
     fma_count: int = 64         # FMAs of the per-nuclide body
-    threshold: int = 24         # best of the sweep (profiles/threshold_sweep_*.md)
+    threshold: int = 32         # best of the sweep with the warp task pool (r02e; the
+                                # static assignment's best was 24, profiles/threshold_sweep_*.md)
     prolog_fma: int = 0         # FMAs of the lookup prolog (expensive task fetch)
     merge_unroll: int = 12      # inner iterations per release, tuned on B200
 
@@ -50,7 +51,7 @@ NEXT1 = RSBench()
 # Fig. 9's XSBench case: an expensive task fetch (2048 FMAs per
 # lookup prolog, ~0.6x the mean inner-loop work of a lookup) -- refilling idle
 # lanes often no longer pays, the best threshold drops
-NEXT1_FETCH = RSBench(prolog_fma=2048, threshold=12)   # best of the sweep
+NEXT1_FETCH = RSBench(prolog_fma=2048, threshold=16)   # best of the pool sweep (static: 12)
 
 
 # (n, mua [1/cm], mus [1/cm], g, d [cm]) -- a synthetic 3-layer tissue slab

@@ -18,7 +18,7 @@ LIB_PATH = os.path.join(HERE, "libsr.so")
 SR_OK, SR_E_INVALID, SR_E_STATE, SR_E_NOMEM, SR_E_CUDA = 0, -1, -2, -3, -4
 PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
 WL_DIVLOOP, WL_COMMONCALL, WL_MCML, WL_PATHTRACE, WL_RSBENCH = 0, 1, 2, 3, 4
-F_SCHED, F_STATIC, F_COARSE, F_NOSPLIT = 1, 2, 4, 8
+F_SCHED, F_STATIC, F_COARSE, F_NOSPLIT, F_MATGROUP = 1, 2, 4, 8, 16
 T_PERTHREAD, T_GRID, T_COUNTERS, T_SCHED, T_SCRATCH = 0, 1, 2, 3, 4
 MAX_LAYERS = 8
 N_COUNTERS = 16

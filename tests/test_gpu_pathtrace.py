@@ -78,7 +78,7 @@ def render(ctx, cfg, mode, T, flags=0, block=0):
 @pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 1), (sr.SPEC_LOOP, 8),
                                     (sr.SPEC_LOOP, 32)])
 @pytest.mark.parametrize("block", [32, 128])
-@pytest.mark.parametrize("flags", [0, sr.F_COARSE, sr.F_NOSPLIT])
+@pytest.mark.parametrize("flags", [0, sr.F_COARSE, sr.F_NOSPLIT, sr.F_MATGROUP])
 def test_render_bit_exact_small(ctx, mode, T, block, flags):
     cfg = I.C4_SMALL
     tris, mat, mats, cam, buf, used = scene(cfg)
@@ -95,6 +95,8 @@ def test_render_full_config_invariants_and_sampled_pixels(ctx):
     b, cb = render(ctx, cfg, sr.PDOM, 0)
     c, cc = render(ctx, cfg, sr.SPEC_LOOP, 16, flags=sr.F_COARSE)
     d, cd = render(ctx, cfg, sr.SPEC_LOOP, 8, flags=sr.F_NOSPLIT)
+    e, ce = render(ctx, cfg, sr.SPEC_LOOP, cfg.threshold, flags=sr.F_MATGROUP)
+    assert np.array_equal(a.view(np.uint32), e.view(np.uint32)) and np.array_equal(ca, ce)
     assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
     assert np.array_equal(a.view(np.uint32), c.view(np.uint32))
     assert np.array_equal(a.view(np.uint32), d.view(np.uint32))

@@ -237,3 +237,73 @@ def test_pool_partial_warp_and_hand_schedule():
     # t=1: lanes 2,3 free -> q4 (2) on lane 2, q5 (5) on lane 3 -> ends at 6
     assert s["STEP"] == (6, 14) and s["LAUNCH"] == (2, 6) and s["ENTRY"] == (1, 3)
     assert s["ADVANCE"] == (2, 4 + 2)   # round 1: all 4 lanes idle; t=1: lanes 2, 3
+
+
+# ------------------------------------------------------------------ task stream (MC dynamic claiming)
+def _stream_ref(ns, W, T, U=1):
+    """the dynamic-claim schedule as an independent set-based event loop"""
+    Q = len(ns)
+    alive, exh, left, q = set(), set(), {}, 0
+    rounds, rel, adv, launch = 0, [0, 0], [0, 0], [0, 0]
+    while True:
+        P = set(alive)
+        R = {l for l in range(W) if l not in alive and l not in exh}
+        if not P and not R:
+            break
+        rounds += 1
+        if len(P) >= T or not R:
+            S = set(P)
+            for _ in range(U):
+                if not S:
+                    break
+                rel[0] += 1
+                rel[1] += len(S)
+                for l in sorted(S):
+                    left[l] -= 1
+                    if left[l] == 0:
+                        alive.discard(l)
+                        S.discard(l)
+        else:
+            adv[0] += 1
+            adv[1] += len(R)
+            got = 0
+            for l in sorted(R):
+                if q >= Q:
+                    exh.add(l)
+                    continue
+                left[l] = int(ns[q])
+                q += 1
+                got += 1
+                alive.add(l)
+            if got:
+                launch[0] += 1
+                launch[1] += got
+    return rounds, tuple(rel), tuple(adv), tuple(launch)
+
+
+def test_stream_matches_reference_and_closed_forms():
+    rng = np.random.default_rng(5)
+    for trial in range(400):
+        W = int(rng.integers(1, 9))
+        Q = int(rng.integers(0, 40))
+        ns = rng.integers(1, 7, Q).astype(np.uint32)
+        T = int(rng.integers(1, W + 1))
+        U = int(rng.integers(1, 4))
+        s = oracle.ws_loopmerge_stream(ns, SPEC_LOOP, T, U=U, W=W)
+        r = _stream_ref(ns, W, T, U)
+        assert (s["rounds"], s["STEP"], s["ADVANCE"], s["LAUNCH"]) == r, (trial, ns, W, T, U)
+        assert s["STEP"][1] == int(ns.sum()) and s["LAUNCH"][1] == Q
+        pd = oracle.ws_loopmerge_stream(ns, PDOM, 0, W=W)
+        assert pd["STEP"][1] == int(ns.sum()) and pd["LAUNCH"][1] == Q
+        assert pd["STEP"][0] == sum(int(ns[b:b + W].max()) for b in range(0, Q, W))
+
+
+def test_stream_events_split_every_step():
+    m = I.C3
+    p = oracle.mc_params(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap)
+    ev, off, ns = oracle.mcml_events_batch(p, 0, 200, I.PRIMARY_SEED)
+    s = oracle.ws_loopmerge_stream(ns, SPEC_LOOP, 32, U=4, ev=np.ascontiguousarray(ev),
+                                   ev_off=off)
+    assert s["STEP"][1] == int(ns.sum()) == len(ev)
+    assert s["STEP_BOUNDARY"][1] + s["STEP_INTERACT"][1] == s["STEP"][1]
+    assert s["STEP_BOUNDARY"][1] == int((np.asarray(ev) & 1).sum())

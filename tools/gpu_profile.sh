@@ -19,6 +19,9 @@ timeout 900 python bench.py > $O/bench_$TAG.json 2> $O/bench_$TAG.err
 M=smsp__thread_inst_executed_per_inst_executed.ratio,smsp__inst_executed.sum,smsp__thread_inst_executed.sum,smsp__thread_inst_executed_pred_on.sum,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__cycles_elapsed.avg.per_second,gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,sm__sass_thread_inst_executed_op_ffma_pred_on.sum,sm__sass_thread_inst_executed_op_ffma2_pred_on.sum,smsp__warps_active.avg.pct_of_peak_sustained_active,launch__registers_per_thread,launch__grid_size,launch__block_size,lts__t_bytes.sum,l1tex__t_bytes.sum
 # every kernel family at its configs[] size (bench launch configuration)
 timeout 1200 ncu --metrics $M --clock-control none -k regex:"divloop|commoncall|mcml|rs_|pt_" --csv --log-file $O/simt_$TAG.csv python tools/one_launch.py > $O/simt_$TAG.log 2>&1
+# the batched-prolog divloop kernels and the static-assignment RSBench kernel
+timeout 600 ncu --metrics $M --clock-control none -k regex:divloop --csv --log-file $O/simt_dlbatch_$TAG.csv python tools/one_launch.py divloop --dl-batch 64 > /dev/null 2>&1
+timeout 600 ncu --metrics $M --clock-control none -k regex:rs_ --csv --log-file $O/simt_rsstatic_$TAG.csv python tools/one_launch.py rsbench --modes spec --rs-flags 2 > /dev/null 2>&1
 # the simulator validation launches (static assignment, the oracle replays every warp)
 timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes pdom,spec --threshold 32 --unroll 1 > /dev/null 2>&1
 timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic8_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes spec --threshold 8 --unroll 1 > /dev/null 2>&1

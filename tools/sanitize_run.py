@@ -70,7 +70,7 @@ if "pathtrace" in what:
     tris, mat, mats, cam = I.cornell_scene(c)
     buf, used = sr.upload_scene(tris, mat, mats, cam)
     n = c.width * c.height
-    for flags in (0, sr.F_SCHED, sr.F_NOSPLIT, sr.F_COARSE):
+    for flags in (0, sr.F_SCHED, sr.F_NOSPLIT, sr.F_COARSE, sr.F_MATGROUP, sr.F_MATGROUP | sr.F_SCHED):
         w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth,
                                   flags=flags)
         run(w, n, 2, sr.PDOM, 0)

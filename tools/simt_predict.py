@@ -61,13 +61,19 @@ def find(costs_all, pattern):
     raise KeyError(pattern)
 
 
-def divloop_warps(mode, T, V=None):
+def divloop_warps(mode, T, V=None, batch=False):
+    """batch: the prolog_batch = 64 kernels -- each valid lane evaluates its
+    conditions in groups of 8 draws at entry (MASKGRP, ceil(iters/8) times)"""
     c = I.C1
     V = c.advance_unroll if V is None else V
     want = oracle.divloop_wants(0, c.n_threads, c.iters, I.PRIMARY_SEED, c.p_u32)
+    groups = (min(c.iters, 64) + 7) // 8
     for w in range(0, c.n_threads, 32):
         ww = want[w:w + 32]
-        yield oracle.ws_divloop(ww, mode, T, V=V if mode == oracle.SPEC_LOOP else 1), len(ww)
+        s = oracle.ws_divloop(ww, mode, T, V=V if mode == oracle.SPEC_LOOP else 1)
+        if batch:
+            s["MASKGRP"] = (groups, groups * len(ww))
+        yield s, len(ww)
 
 
 def commoncall_warps(mode):
@@ -92,13 +98,42 @@ def mcml_warps(mode, T, n_threads=MC_VALIDATION["n_threads"], iters=MC_VALIDATIO
         yield oracle.ws_loopmerge_raw(ns[ids], ev, off[ids].ravel(), mode, T, U=U), len(lanes)
 
 
-def rsbench_warps(mode, T, U=None):
+def rsbench_warps(mode, T, U=None, pool=False):
+    """pool: the default warp task pool (SPEC); else lane l runs thread l's lookups"""
     c = I.NEXT1
     U = c.merge_unroll if U is None else U
     _, _, trips = oracle.rsbench(0, c.n_threads, c.iters, I.PRIMARY_SEED, fma_count=0, trips=True)
     for w in range(0, c.n_threads, 32):
         tr = trips[w:w + 32]
-        yield oracle.ws_loopmerge(tr, mode, T, U=U if mode == oracle.SPEC_LOOP else 1), len(tr)
+        if pool and mode == oracle.SPEC_LOOP:
+            s = oracle.ws_loopmerge_pool(tr, T, U=U)
+            s["PERK"] = (c.iters, c.iters * len(tr))   # the in-order per-thread sum
+            yield s, len(tr)
+        else:
+            yield oracle.ws_loopmerge(tr, mode, T, U=U if mode == oracle.SPEC_LOOP else 1), len(tr)
+
+
+# the bench launch of configs[2] (dynamic claiming): a persistent grid of
+# 2 x 148 CTAs of 640 threads = 5920 warps, each taking ~10^7 / 5920 photons in
+# chunks from one counter.  Which photons a warp gets depends on timing; their
+# step counts are i.i.d., so each sampled warp replays a stream of consecutive
+# photon ids of the same length (one drain at the end, as on the GPU).
+MC_DYN = dict(warps=5920, sample_warps=48)
+
+
+def mcml_dyn_warps(mode, T, U=None, photons=None, sample=None):
+    m = I.C3
+    U = m.merge_unroll if U is None else U
+    photons = photons or m.n_photons
+    sample = sample or MC_DYN["sample_warps"]
+    q = photons // MC_DYN["warps"]
+    p = oracle.mc_params(m.layers, m.n_above, m.n_below, m.dr, m.dz, m.nr, m.nz, m.step_cap)
+    ev, off, ns = oracle.mcml_events_batch(p, 0, q * sample, I.PRIMARY_SEED)
+    ev = np.ascontiguousarray(ev)
+    for w in range(sample):
+        sl = slice(w * q, (w + 1) * q)
+        yield oracle.ws_loopmerge_stream(ns[sl], mode, T, U=U if mode == oracle.SPEC_LOOP else 1,
+                                         ev=ev, ev_off=off[sl]), 32
 
 
 CASES = {
@@ -112,8 +147,25 @@ CASES = {
     "mcml_spec_static(T=32,U=4)": (r"mcml_specILb0ELb0ELb1",
                                    lambda: mcml_warps(oracle.SPEC_LOOP, 32, U=4)),
     "rs_pdom": (r"rs_pdomILi8ELi0ELb0", lambda: rsbench_warps(oracle.PDOM, 0)),
-    "rs_spec(T=24)": (r"rs_specILi8ELi0ELb0", lambda: rsbench_warps(oracle.SPEC_LOOP, 24)),
+    f"rs_spec(T={I.NEXT1.threshold})": (
+        r"rs_specILi8ELi0ELb0ELb1E",
+        lambda: rsbench_warps(oracle.SPEC_LOOP, I.NEXT1.threshold, pool=True)),
+    f"rs_spec_static(T={I.NEXT1.threshold})": (
+        r"rs_specILi8ELi0ELb0ELb0E", lambda: rsbench_warps(oracle.SPEC_LOOP, I.NEXT1.threshold)),
+    "divloop_pdom_batch": (r"divloop_pdom_batchILi125ELb0",
+                           lambda: divloop_warps(oracle.PDOM, 0, batch=True)),
+    "divloop_spec_batch(T=16)": (r"divloop_spec_batchILi125ELb0",
+                                 lambda: divloop_warps(oracle.SPEC_LOOP, 16, batch=True)),
+    "mcml_pdom": (r"mcml_pdomILb1ELb0ELb1", lambda: mcml_dyn_warps(oracle.PDOM, 0)),
+    "mcml_spec(T=32)": (r"mcml_specILb1ELb0ELb1", lambda: mcml_dyn_warps(oracle.SPEC_LOOP, 32)),
 }
+
+
+def inst_scale(label):
+    """the sampled-warp cases predict instructions for sample_warps of the launch"""
+    if label in ("mcml_pdom", "mcml_spec(T=32)"):
+        return MC_DYN["warps"] / MC_DYN["sample_warps"]
+    return 1.0
 
 
 def main():
@@ -125,8 +177,9 @@ def main():
         p = predict(find(costs, pat), gen())
         m = measured.get(label, {})
         rows[label] = dict(predicted=p["simt"], measured=m.get("simt_efficiency"),
-                           predicted_inst=p["inst"], measured_inst=m.get("inst"),
-                           predicted_thread_inst=p["thread_inst"],
+                           predicted_inst=p["inst"] * inst_scale(label),
+                           measured_inst=m.get("inst"),
+                           predicted_thread_inst=p["thread_inst"] * inst_scale(label),
                            measured_thread_inst=m.get("thread_inst"),
                            costs=find(costs, pat))
         if m.get("simt_efficiency") is not None:

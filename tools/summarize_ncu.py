@@ -20,9 +20,15 @@ OUT = os.path.join(ROOT, "gpurun_out")
 PROF = os.path.join(ROOT, "profiles")
 
 # launch order of tools/one_launch.py (default: every family, pdom then spec)
+sys.path.insert(0, ROOT)
+from paper_conf_cgo_damanijskymg20_b200 import inputs as _I  # noqa: E402
+
+_TRS = _I.NEXT1.threshold
 LABELS_ALL = ["divloop_pdom", "divloop_spec(T=16)", "commoncall_pdom", "commoncall_spec",
-              "mcml_pdom", "mcml_spec(T=32)", "rs_pdom", "rs_spec(T=24)", "pt_pdom",
-              "pt_spec(T=12)"]
+              "mcml_pdom", "mcml_spec(T=32)", "rs_pdom", f"rs_spec(T={_TRS})", "pt_pdom",
+              f"pt_spec(T={_I.C4.threshold})"]
+LABELS_DLBATCH = ["divloop_pdom_batch", "divloop_spec_batch(T=16)"]
+LABELS_RSSTATIC = [f"rs_spec_static(T={_TRS})"]
 LABELS_MCSTATIC = ["mcml_pdom_static", "mcml_spec_static(T=32)"]
 LABELS_MCSTATIC8 = ["mcml_spec_static(T=8)"]
 LABELS_MCSTATICU4 = ["mcml_spec_static(T=32,U=4)"]
@@ -98,7 +104,9 @@ def main():
     for fname, labels in ((f"simt_{tag}.csv", LABELS_ALL),
                           (f"simt_mcstatic_{tag}.csv", LABELS_MCSTATIC),
                           (f"simt_mcstatic8_{tag}.csv", LABELS_MCSTATIC8),
-                          (f"simt_mcstaticu4_{tag}.csv", LABELS_MCSTATICU4)):
+                          (f"simt_mcstaticu4_{tag}.csv", LABELS_MCSTATICU4),
+                          (f"simt_dlbatch_{tag}.csv", LABELS_DLBATCH),
+                          (f"simt_rsstatic_{tag}.csv", LABELS_RSSTATIC)):
         path = os.path.join(OUT, fname)
         if not os.path.exists(path):
             continue

@@ -29,6 +29,8 @@ ap.add_argument("--defer", type=int, default=0, help="MCML boundary defer thresh
 ap.add_argument("--static", action="store_true", help="MCML static photon assignment (F_STATIC)")
 ap.add_argument("--iters", type=int, default=0, help="MCML photons per lane (default configs[2])")
 ap.add_argument("--prolog", type=int, default=0, help="RSBench prolog FMAs (expensive task fetch)")
+ap.add_argument("--batch", type=int, default=0, help="divloop prolog_batch (0 or 64)")
+ap.add_argument("--unrolls", default="", help="comma list: sweep the merge unroll too")
 a = ap.parse_args()
 Ts = [int(x) for x in a.thresholds.split(",")]
 blocks = [int(x) for x in a.blocks.split(",")]
@@ -89,7 +91,8 @@ if "divloop" in a.what:
     c = I.C1
     res = []
     for b in blocks:
-        w = sr.divloop_workload(c.p_u32, c.fma_count, block=b, advance=a.unroll)
+        w = sr.divloop_workload(c.p_u32, c.fma_count, block=b, advance=a.unroll, batch=a.batch,
+                                flags=a.flags)
         ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
             def run():
@@ -105,12 +108,14 @@ if "divloop" in a.what:
 if "rsbench" in a.what:
     c = I.NEXT1
     res = []
-    for b in blocks:
-        w = sr.rsbench_workload(c.fma_count, block=b, prolog_fma=a.prolog, unroll=a.unroll)
+    Us = [int(x) for x in a.unrolls.split(",")] if a.unrolls else [a.unroll]
+    for b, U in [(b, U) for b in blocks for U in Us]:
+        w = sr.rsbench_workload(c.fma_count, block=b, prolog_fma=a.prolog, unroll=U, flags=a.flags)
         ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
-        for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
+        for mode, T in ([(sr.PDOM, 0)] if U == Us[0] else []) + [(sr.SPEC_LOOP, t) for t in Ts]:
             t = timed(lambda: sr.sr_run(w, c.n_threads, c.iters, seed, mode, T), a.reps)
-            r = dict(block=b, mode="pdom" if mode == sr.PDOM else "spec", T=T, ms=t,
+            r = dict(block=b, mode="pdom" if mode == sr.PDOM else "spec", T=T, ms=t, unroll=U,
+                     flags=a.flags,
                      lookups_per_s=c.n_threads * c.iters / (t * 1e-3), launch=sr.sr_last_launch())
             r.update(eff(w, c.n_threads, c.iters, mode, T))
             res.append(r)
