@@ -180,11 +180,11 @@ __global__ void __launch_bounds__(SR_RS_MAXT) rs_spec(const RsArgs a) {
         const uint32_t q = qnext + (uint32_t)__popc(R & lanemask_lt());
         go = go && q < pool;
         if (go) {
-          own = nv == 32u ? (q & 31u) : q % nv;
+          own = nv == 32u ? (q & 31u) : q % nv;  // @sr-region LAUNCH
           k = nv == 32u ? (q >> 5) : q / nv;
           t = a.t0 + (g & ~31ull) + own;
         }
-        qnext = min(pool, qnext + (uint32_t)__popc(R));
+        qnext = min(pool, qnext + (uint32_t)__popc(R));  // @sr-region ADVANCE:full
       }
       if (go) {
         const uint4 u = draw(k, kTagRs, t, a.keys);  // @sr-region LAUNCH
@@ -204,6 +204,7 @@ __global__ void __launch_bounds__(SR_RS_MAXT) rs_spec(const RsArgs a) {
   if constexpr (POOL) {  // @sr-region ENTRY:full
     __syncwarp();
     if (valid) {  // this thread's lookups in program order
+#pragma unroll 1  // one trip per lookup (the simulator's PERK count)
       for (uint32_t kk = 0; kk < a.iters; ++kk) acc = acc + xw[kk * 32u + lane_id()];  // @sr-region PERK:full
       nucs = nw[lane_id()];  // @sr-region ENTRY:full
     }

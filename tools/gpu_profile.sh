@@ -39,7 +39,9 @@ timeout 300 $SC -k regex:mcml -o $O/src_mc_spec32_$TAG $OL $MCS --modes spec --t
 timeout 300 $SC -k regex:mcml -o $O/src_mc_spec8_$TAG $OL $MCS --modes spec --threshold 8 --unroll 1 > /dev/null 2>&1
 timeout 300 $SC -k regex:mcml -o $O/src_mc_spec32u4_$TAG $OL $MCS --modes spec --threshold 32 --unroll 4 > /dev/null 2>&1
 # full captures of the path tracer kernels (PDOM and the default split merge)
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:pt_ -c 2 -o $O/prof_pt_$TAG $OL pathtrace > $O/prof_pt_$TAG.log 2>&1
+# (one kernel per process: a second full capture in the same process came back mostly NaN)
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:pt_pdom -c 1 -o $O/prof_ptpdom_$TAG $OL pathtrace --modes pdom > $O/prof_pt_$TAG.log 2>&1
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:pt_spec -c 1 -o $O/prof_ptspec_$TAG $OL pathtrace --modes spec >> $O/prof_pt_$TAG.log 2>&1
 # launch list of one short bench run (shares, not absolutes)
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-configs > $O/launches_$TAG.log 2>&1
 # full captures of the dominant kernel (and its PDOM baseline), at 2M photons

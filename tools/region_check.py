@@ -35,7 +35,7 @@ import simt_predict as sp  # noqa: E402
 # label -> report key (one single-launch report each)
 REPORTS = {
     "divloop_pdom": "divloop_pdom", "divloop_spec(T=16)": "divloop_spec",
-    "rs_pdom": "rs_pdom", "rs_spec(T=24)": "rs_spec",
+    "rs_pdom": "rs_pdom", "rs_spec(T=32)": "rs_spec",
     "mcml_pdom_static": "mc_pdom", "mcml_spec_static(T=32)": "mc_spec32",
     "mcml_spec_static(T=8)": "mc_spec8", "mcml_spec_static(T=32,U=4)": "mc_spec32u4",
 }
