@@ -101,9 +101,11 @@ typedef struct {
                           one draw at a time, as Fig. 2(a) is written; 64 = a lane
                           evaluates the divergent conditions of up to 64 of its
                           iterations together (independent counters, ILP) into a
-                          64-bit mask, and redraws only the iterations that call
-                          Expensive() (reading Q5').  Other values: SR_E_INVALID.
-                          Results and schedule counters are identical.          */
+                          64-bit mask and keeps the Expensive() arguments of the
+                          iterations that call it in shared memory (256 bytes per
+                          thread; needs block_threads <= 512) (reading Q5').
+                          Other values: SR_E_INVALID.  Results and schedule
+                          counters are identical.                              */
 } sr_divloop_params;
 
 typedef struct {

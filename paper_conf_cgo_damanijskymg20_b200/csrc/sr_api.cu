@@ -71,6 +71,9 @@ std::string check_workload(const sr_workload* w, uint64_t n_threads) {
       if (w->divloop.fma_count % 8 != 0) return "divloop.fma_count must be a multiple of 8";
       if (w->divloop.prolog_batch > 1 && w->divloop.prolog_batch != 64)
         return "divloop.prolog_batch must be 0, 1 or 64";
+      if (w->divloop.prolog_batch == 64 && w->block_threads > 512)
+        return "divloop.prolog_batch = 64 needs block_threads <= 512 (64 shared-memory floats "
+               "per thread)";
       if (n_threads > (1ull << 40)) return "n_threads too large";
       return "";
     case SR_WL_COMMONCALL:

@@ -98,6 +98,9 @@ def test_run_validation_before_state():
         with pytest.raises(sr.SRError) as e:
             sr.sr_run(bad, 64, 1, 1, sr.PDOM, 0)
         assert e.value.code == sr.SR_E_INVALID and "prolog_batch" in str(e.value)
+    with pytest.raises(sr.SRError) as e:
+        sr.sr_run(sr.divloop_workload(batch=64, block=1024), 64, 1, 1, sr.PDOM, 0)
+    assert e.value.code == sr.SR_E_INVALID and "block_threads <= 512" in str(e.value)
 
 
 def test_mcml_param_validation():

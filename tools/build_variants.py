@@ -26,6 +26,8 @@ VARIANTS = {
     "libsr_ch128.so": ["SR_MC_CHUNK=128"],
     "libsr_pt9.so": ["SR_PT_MINB_SPEC=9", "SR_PT_MINB_PDOM=9"],
     "libsr_pt10.so": ["SR_PT_MINB_SPEC=10", "SR_PT_MINB_PDOM=10"],
+    "libsr_pt8.so": ["SR_PT_MINB_SPEC=8", "SR_PT_MINB_PDOM=8"],
+    "libsr_pt7.so": ["SR_PT_MINB_SPEC=7", "SR_PT_MINB_PDOM=7"],
 }
 if __name__ == "__main__":
     names = sys.argv[1:] or list(VARIANTS)

@@ -25,6 +25,8 @@ ap.add_argument("--unroll", type=int, default=I.C3.merge_unroll,
                 help="MCML merge unroll (default: the bench's, configs[2])")
 ap.add_argument("--pt-flags", type=int, default=0, help="extra PATHTRACE flags (F_NOSPLIT = 8)")
 ap.add_argument("--dl-batch", type=int, default=0, help="divloop prolog_batch (0 or 64)")
+ap.add_argument("--dl-threads", type=int, default=0, help="divloop threads (default configs[0])")
+ap.add_argument("--dl-fma", type=int, default=-1, help="divloop FMAs per Expensive (default configs[0])")
 ap.add_argument("--rs-flags", type=int, default=0, help="extra RSBENCH flags (F_STATIC = 2)")
 a = ap.parse_args()
 modes = a.modes.split(",")
@@ -32,10 +34,12 @@ ctx = sr.Context.create(0, 1 << 20)
 seed = I.PRIMARY_SEED
 if "divloop" in a.what:
     c = I.C1
-    w = sr.divloop_workload(c.p_u32, c.fma_count, advance=c.advance_unroll, batch=a.dl_batch)
-    ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
+    nth = a.dl_threads or c.n_threads
+    w = sr.divloop_workload(c.p_u32, c.fma_count if a.dl_fma < 0 else a.dl_fma,
+                            advance=c.advance_unroll, batch=a.dl_batch)
+    ctx.ensure(sr.sr_workspace_bytes(w, nth))
     for md in modes:
-        sr.sr_run(w, c.n_threads, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
+        sr.sr_run(w, nth, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,
                   0 if md == "pdom" else c.threshold)
 if "commoncall" in a.what:
     c = I.C2
