@@ -20,7 +20,7 @@ namespace sr {
 namespace {
 
 constexpr int kBins = 16;
-constexpr int kLeafMax = (int)kPtLeafMax;   // a leaf never holds more than this many triangles
+constexpr int kLeafMax = 8;   // a leaf never holds more than this many triangles
 constexpr int kLeafMin = 2;   // ranges this small always become leaves
 
 struct Box {
@@ -160,7 +160,7 @@ float pad_lo(float v) { return std::nextafter(v - std::fabs(v) * 1e-5f - 1e-6f, 
 float pad_hi(float v) { return std::nextafter(v + std::fabs(v) * 1e-5f + 1e-6f, INFINITY); }
 
 size_t image_bound(uint32_t n_tris, uint32_t n_mats) {
-  const size_t nodes = std::max<size_t>(n_tris, 1);   // >= the binary tree's inner nodes
+  const size_t nodes = std::max<size_t>(n_tris, 1);
   return sizeof(PtHeader) + nodes * sizeof(PtNode) + (size_t)n_tris * sizeof(PtTri) +
          (size_t)n_mats * sizeof(PtMat);
 }
@@ -170,8 +170,7 @@ size_t image_bound(uint32_t n_tris, uint32_t n_mats) {
 std::string check_scene_inputs(const float* tris, const uint32_t* mat, uint32_t n_tris,
                                const float* mats, uint32_t n_mats, const float* cam) {
   if (n_tris == 0) return "n_tris must be >= 1";
-  if (n_tris >= kPtLeafFirstMax)
-    return "n_tris must be < 2^28 (traversal-stack leaf entries pack first << 3 | count - 1)";
+  if (n_tris >= (1u << 31)) return "n_tris must be < 2^31 (BVH references are int32)";
   if (!tris || !mat || !mats || !cam) return "NULL input array";
   if (n_mats == 0) return "n_mats must be >= 1";
   for (size_t i = 0; i < 9 * (size_t)n_tris; ++i)
@@ -219,80 +218,68 @@ static int build_scene(const char* fn, bool to_device, const float* tris, const 
   }
   B.build();
 
-  // collapse the binary tree into four-wide nodes: a node starts from its two
-  // binary children and keeps replacing the inner child of largest surface area
-  // by that child's two children (in place, so siblings stay in spatial order)
-  // until it has four children or only leaves; flattened in pre-order
-  auto children4 = [&](int b) {
-    std::vector<int> ch;
-    if (B.nodes[b].count > 0) { ch.push_back(b); return ch; }   // a leaf root: one leaf child
-    ch = {B.nodes[b].left, B.nodes[b].right};
-    while (ch.size() < kPtWide) {
-      int best = -1;
-      double area = -1.0;
-      for (size_t k = 0; k < ch.size(); ++k) {
-        const BNode& c = B.nodes[ch[k]];
-        if (c.count == 0 && c.box.area() > area) { area = c.box.area(); best = (int)k; }
-      }
-      if (best < 0) break;
-      const int c = ch[best];
-      ch[best] = B.nodes[c].left;
-      ch.insert(ch.begin() + best + 1, B.nodes[c].right);
-    }
-    return ch;
-  };
-  std::vector<PtNode> nodes;
-  std::vector<uint32_t> need;   // per node4: deepest stack below it (entries)
+  // flatten: one PtNode per inner build node, pre-order; leaves fold into refs
+  std::vector<int> out_of(B.nodes.size(), -1);
+  std::vector<int> order;
   {
-    struct Item { int b, out; };
-    std::vector<Item> st{{0, 0}};
-    nodes.emplace_back();
-    std::vector<std::vector<int>> kids;   // child node4 indices of each node4, for `need`
-    kids.emplace_back();
+    std::vector<int> st{0};
     while (!st.empty()) {
-      const Item it = st.back();
+      const int n = st.back();
       st.pop_back();
-      const std::vector<int> ch = children4(it.b);
-      PtNode o;
-      std::vector<std::pair<int, int>> inner;   // (slot, binary node) of inner children
-      for (uint32_t k = 0; k < kPtWide; ++k) {
-        if (k >= ch.size()) {
-          o.lox[k] = o.loy[k] = o.loz[k] = INFINITY;
-          o.hix[k] = o.hiy[k] = o.hiz[k] = -INFINITY;
-          o.ref[k] = -1;
-          o.cnt[k] = 0;
-          continue;
-        }
-        const BNode& c = B.nodes[ch[k]];
-        o.lox[k] = pad_lo(c.box.lo[0]); o.loy[k] = pad_lo(c.box.lo[1]); o.loz[k] = pad_lo(c.box.lo[2]);
-        o.hix[k] = pad_hi(c.box.hi[0]); o.hiy[k] = pad_hi(c.box.hi[1]); o.hiz[k] = pad_hi(c.box.hi[2]);
-        if (c.count > 0) { o.ref[k] = c.start; o.cnt[k] = c.count; }
-        else { o.ref[k] = -1; o.cnt[k] = 0; inner.push_back({(int)k, ch[k]}); }
+      if (B.nodes[n].count > 0 && n != 0) continue;
+      out_of[n] = (int)order.size();
+      order.push_back(n);
+      if (B.nodes[n].count == 0) {
+        st.push_back(B.nodes[n].right);
+        st.push_back(B.nodes[n].left);
       }
-      // pre-order: children are numbered in slot order, pushed in reverse
-      std::vector<int> idx;
-      for (const auto& [slot, b] : inner) {
-        o.ref[slot] = (int32_t)nodes.size() + (int32_t)idx.size();
-        idx.push_back(o.ref[slot]);
-      }
-      nodes[it.out] = o;
-      kids[it.out] = idx;
-      for (size_t k = 0; k < inner.size(); ++k) { nodes.emplace_back(); kids.emplace_back(); }
-      for (size_t k = inner.size(); k-- > 0;) st.push_back({inner[k].second, idx[k]});
-    }
-    // the numbering above is breadth-per-node (siblings contiguous), children after
-    // their parent; the stack bound: a visit keeps its nearest hit child and pushes
-    // every other hit child (inner or leaf), so a ray holds at most
-    // sum over its root path of (children - 1) entries
-    need.assign(nodes.size(), 0);
-    for (size_t i = nodes.size(); i-- > 0;) {
-      uint32_t nch = 0, below = 0;
-      for (uint32_t k = 0; k < kPtWide; ++k) nch += nodes[i].ref[k] >= 0 ? 1u : 0u;
-      for (int c : kids[i]) below = std::max(below, need[c]);
-      need[i] = (nch > 0 ? nch - 1 : 0) + below;
     }
   }
-  const uint32_t stack_need = need.empty() ? 0u : need[0];
+  std::vector<PtNode> nodes(order.size());
+  auto set_child = [&](PtNode& o, int slot, int c) {
+    float* lo = slot ? o.b1lo : o.b0lo;
+    float* hi = slot ? o.b1hi : o.b0hi;
+    int32_t& ref = slot ? o.ref1 : o.ref0;
+    int32_t& cnt = slot ? o.cnt1 : o.cnt0;
+    if (c < 0) {
+      for (int k = 0; k < 3; ++k) { lo[k] = INFINITY; hi[k] = -INFINITY; }
+      ref = -1;
+      cnt = 0;
+      return;
+    }
+    const BNode& b = B.nodes[c];
+    for (int k = 0; k < 3; ++k) { lo[k] = pad_lo(b.box.lo[k]); hi[k] = pad_hi(b.box.hi[k]); }
+    if (b.count > 0) { ref = b.start; cnt = b.count; }
+    else { ref = out_of[c]; cnt = 0; }
+  };
+  for (size_t i = 0; i < order.size(); ++i) {
+    const BNode& b = B.nodes[order[i]];
+    if (b.count > 0) {           // the root itself is a leaf: wrap it
+      set_child(nodes[i], 0, order[i]);
+      set_child(nodes[i], 1, -1);
+    } else {
+      set_child(nodes[i], 0, b.left);
+      set_child(nodes[i], 1, b.right);
+    }
+  }
+
+  // traversal stack bound: a visit pushes at most one entry (the farther of
+  // two inner children), so a ray holds at most (inner nodes on its root path
+  // - 1) entries
+  uint32_t stack_need = 0;
+  {
+    std::vector<std::pair<int, uint32_t>> st{{0, 0u}};
+    while (!st.empty()) {
+      const auto [i, d] = st.back();
+      st.pop_back();
+      stack_need = std::max(stack_need, d);
+      const PtNode& o = nodes[i];
+      const bool in0 = o.ref0 >= 0 && o.cnt0 == 0, in1 = o.ref1 >= 0 && o.cnt1 == 0;
+      const uint32_t dd = d + ((in0 && in1) ? 1u : 0u);
+      if (in0) st.push_back({o.ref0, dd});
+      if (in1) st.push_back({o.ref1, dd});
+    }
+  }
 
   std::vector<unsigned char> img(bound, 0);
   PtHeader h{};

@@ -104,6 +104,17 @@ struct Stats {
 // one scalar load per field (the structs are 4-byte aligned, so the compiler
 // would not vectorise them itself; the image keeps every record 16-byte
 // aligned: 128-byte header, 64-byte nodes, 48-byte triangles).
+__device__ __forceinline__ PtNode load_node(const PtNode* base, int32_t i) {
+  const float4* q = reinterpret_cast<const float4*>(base + i);
+  const float4 x = __ldg(q), y = __ldg(q + 1), z = __ldg(q + 2);
+  const int4 w = __ldg(reinterpret_cast<const int4*>(q + 3));
+  PtNode n;
+  n.b0lo[0] = x.x; n.b0lo[1] = x.y; n.b0lo[2] = x.z; n.b0hi[0] = x.w;
+  n.b0hi[1] = y.x; n.b0hi[2] = y.y; n.b1lo[0] = y.z; n.b1lo[1] = y.w;
+  n.b1lo[2] = z.x; n.b1hi[0] = z.y; n.b1hi[1] = z.z; n.b1hi[2] = z.w;
+  n.ref0 = w.x; n.cnt0 = w.y; n.ref1 = w.z; n.cnt1 = w.w;
+  return n;
+}
 __device__ __forceinline__ PtTri load_tri(const PtTri* base, int32_t i) {
   const float4* q = reinterpret_cast<const float4*>(base + i);
   const float4 x = __ldg(q), y = __ldg(q + 1);
@@ -123,9 +134,18 @@ __device__ __forceinline__ PtMat load_mat(const PtMat* base, uint32_t i) {
   return m;
 }
 
-// Box test (trav_node): conservative slab test against a padded box -- accept
-// when the ray's parametric interval [tmin, tbest] can touch the box (slack
-// 1e-5 relative).
+// Conservative slab test against a padded box: accept when the ray's
+// parametric interval [tmin, tbest] can touch the box (slack 1e-5 relative).
+__device__ __forceinline__ bool box_hit(const float* lo, const float* hi, V3 o, V3 inv, float tb,
+                                        float& tnear) {
+  const float tx0 = (lo[0] - o.x) * inv.x, tx1 = (hi[0] - o.x) * inv.x;
+  const float ty0 = (lo[1] - o.y) * inv.y, ty1 = (hi[1] - o.y) * inv.y;
+  const float tz0 = (lo[2] - o.z) * inv.z, tz1 = (hi[2] - o.z) * inv.z;
+  const float tn = fmaxf(fmaxf(fminf(tx0, tx1), fminf(ty0, ty1)), fmaxf(fminf(tz0, tz1), 0.0f));
+  const float tf = fminf(fminf(fmaxf(tx0, tx1), fmaxf(ty0, ty1)), fmaxf(tz0, tz1));
+  tnear = tn;
+  return tn * (1.0f - 1e-5f) <= tf * (1.0f + 1e-5f) && tn * (1.0f - 1e-5f) <= tb;
+}
 
 // Moller-Trumbore exactly as the oracle (e1, e2 precomputed with the same
 // binary32 subtractions).
@@ -155,16 +175,10 @@ __device__ __forceinline__ void tri_test(const PtTri& T, int32_t at, V3 o, V3 d,
   }
 }
 
-// Resumable BVH traversal over the four-wide tree.  The traversal state is one
-// pending entry -- an inner node (tr.node >= 0) or a leaf's triangle range
-// (tr.na > 0) -- plus a stack of further entries.  Visiting a node tests its four
-// child boxes; the nearest hit child (inner or leaf) becomes the pending entry and
-// the other hit children are pushed farthest first, so they pop nearest first;
-// no hit child: pop.  A leaf entry's triangles are tested in order, then the next
-// entry pops.  closest_hit() runs trav_step (one entry: a node visit or a whole
-// leaf) to completion; the node-granularity Loop Merge kernels interleave single
-// entries of different lanes' rays, and the split merge runs node visits
-// (trav_node) and single triangle tests (trav_leaf) as separate regions.
+// Resumable BVH traversal: one call of trav_step visits one node (its two
+// child boxes, the triangles of child leaves, push/pop).  closest_hit() runs
+// it to completion; the node-granularity Loop Merge kernel interleaves single
+// steps of different lanes' rays.
 //
 // The traversal stack lives in shared memory, one column per thread
 // (entry i of thread t at smem[i * blockDim + t]: consecutive lanes hit
@@ -175,10 +189,12 @@ struct Trav {
   float tb;
   int32_t ib;       // original index of the closest triangle so far (-1: none)
   uint32_t mb, slot;
-  int32_t node;     // pending inner node, or -1
+  int32_t node;
   int32_t sp;
-  int32_t la;       // pending leaf range: triangles [la, la + na)
-  uint32_t na;
+  // split merge (default): leaf ranges found by the last node visit, tested later by
+  // trav_leaf (current range la/na, queued range lb/nb)
+  int32_t la, lb;
+  uint32_t na, nb;
 };
 
 extern __shared__ int32_t pt_stack_smem[];
@@ -186,25 +202,6 @@ extern __shared__ int32_t pt_stack_smem[];
 // so no per-lane pointer is kept in registers)
 __device__ __forceinline__ int32_t& stk(int32_t i) {
   return pt_stack_smem[(uint32_t)i * blockDim.x + threadIdx.x];
-}
-
-__device__ __forceinline__ int32_t leaf_entry(int32_t first, int32_t cnt) {
-  return ~((first << 3) | (cnt - 1));
-}
-// make entry e pending (e >= 0: inner node; e < 0: a leaf)
-__device__ __forceinline__ void set_pending(Trav& tr, int32_t e) {
-  if (e >= 0) {
-    tr.node = e;
-    tr.na = 0u;
-  } else {
-    tr.node = -1;
-    tr.la = (~e) >> 3;
-    tr.na = (uint32_t)((~e) & 7) + 1u;
-  }
-}
-__device__ __forceinline__ void pop_pending(Trav& tr) {
-  if (tr.sp > 0) set_pending(tr, stk(--tr.sp));
-  else { tr.node = -1; tr.na = 0u; }
 }
 
 __device__ __forceinline__ void trav_begin(Trav& tr, V3 d) {
@@ -215,94 +212,90 @@ __device__ __forceinline__ void trav_begin(Trav& tr, V3 d) {
   tr.slot = 0;
   tr.node = 0;
   tr.sp = 0;
-  tr.la = 0;
-  tr.na = 0u;
+  tr.na = 0;
+  tr.nb = 0;
 }
 
-// visits tr.node: four box tests, then the nearest hit child becomes pending and
-// the others go on the stack (farthest first); no hit: pop
-__device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats& st) {
-  // the four slab tests axis by axis (the node's rows are loaded as needed, so
-  // only a running [near, far] pair per child stays live): the same fminf / fmaxf
-  // expression as box_hit, operand for operand
-  const float4* q = reinterpret_cast<const float4*>(a.nodes + tr.node);
+// returns false when the traversal is finished
+__device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
+  const PtNode N = load_node(a.nodes, tr.node);
   ++st.nodes;
-  float t[4], f[4];
-  {
-    const float4 lo = __ldg(q), hi = __ldg(q + 3);
-    const float l[4] = {lo.x, lo.y, lo.z, lo.w}, h[4] = {hi.x, hi.y, hi.z, hi.w};
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const float t0 = (l[k] - o.x) * tr.inv.x, t1 = (h[k] - o.x) * tr.inv.x;
-      t[k] = fminf(t0, t1);
-      f[k] = fmaxf(t0, t1);
+  float tn0, tn1;
+  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0);
+  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1);
+  // leaves: test their triangles now; inner children: descend / push
+  if (h0 && N.cnt0 > 0) {
+    for (int32_t k = 0; k < N.cnt0; ++k) {
+      tri_test(load_tri(a.tris, N.ref0 + k), N.ref0 + k, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
+      ++st.tests;
     }
   }
-  {
-    const float4 lo = __ldg(q + 1), hi = __ldg(q + 4);
-    const float l[4] = {lo.x, lo.y, lo.z, lo.w}, h[4] = {hi.x, hi.y, hi.z, hi.w};
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const float t0 = (l[k] - o.y) * tr.inv.y, t1 = (h[k] - o.y) * tr.inv.y;
-      t[k] = fmaxf(t[k], fminf(t0, t1));
-      f[k] = fminf(f[k], fmaxf(t0, t1));
+  if (h1 && N.cnt1 > 0) {
+    for (int32_t k = 0; k < N.cnt1; ++k) {
+      tri_test(load_tri(a.tris, N.ref1 + k), N.ref1 + k, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
+      ++st.tests;
     }
   }
-  {
-    const float4 lo = __ldg(q + 2), hi = __ldg(q + 5);
-    const float l[4] = {lo.x, lo.y, lo.z, lo.w}, h[4] = {hi.x, hi.y, hi.z, hi.w};
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const float t0 = (l[k] - o.z) * tr.inv.z, t1 = (h[k] - o.z) * tr.inv.z;
-      t[k] = fmaxf(t[k], fmaxf(fminf(t0, t1), 0.0f));
-      f[k] = fminf(f[k], fmaxf(t0, t1));
-    }
+  const bool in0 = h0 && N.cnt0 == 0, in1 = h1 && N.cnt1 == 0;
+  int32_t next = -1;
+  if (in0 && in1) {
+    const bool first0 = tn0 <= tn1;
+    next = first0 ? N.ref0 : N.ref1;
+    if ((uint32_t)tr.sp < a.stack_cap) stk(tr.sp++) = first0 ? N.ref1 : N.ref0;
+  } else if (in0) {
+    next = N.ref0;
+  } else if (in1) {
+    next = N.ref1;
   }
-  const int4 rf = __ldg(reinterpret_cast<const int4*>(q + 6));
-  const int4 cn = __ldg(reinterpret_cast<const int4*>(q + 7));
-  const int32_t ref[4] = {rf.x, rf.y, rf.z, rf.w}, cnt[4] = {cn.x, cn.y, cn.z, cn.w};
-  int32_t e[4];
-#pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    const bool h = ref[k] >= 0 && t[k] * (1.0f - 1e-5f) <= f[k] * (1.0f + 1e-5f) &&
-                   t[k] * (1.0f - 1e-5f) <= tr.tb;
-    if (!h) t[k] = INFINITY;
-    e[k] = !h ? INT32_MIN : (cnt[k] > 0 ? leaf_entry(ref[k], cnt[k]) : ref[k]);
+  if (next < 0) {
+    if (tr.sp == 0) return false;
+    next = stk(--tr.sp);
   }
-  // sort the four (t, entry) pairs by t (a 5-comparator network; misses carry
-  // t = +inf and sort last)
-#define SR_CSWAP(i, j)                                                   \
-  if (t[j] < t[i]) {                                                     \
-    const float tt = t[i]; t[i] = t[j]; t[j] = tt;                       \
-    const int32_t ee = e[i]; e[i] = e[j]; e[j] = ee;                     \
-  }
-  SR_CSWAP(0, 1) SR_CSWAP(2, 3) SR_CSWAP(0, 2) SR_CSWAP(1, 3) SR_CSWAP(1, 2)
-#undef SR_CSWAP
-  // push hit children 3, 2, 1 (farthest first), keep child 0
-#pragma unroll
-  for (int k = 3; k >= 1; --k)
-    if (e[k] != INT32_MIN && (uint32_t)tr.sp < a.stack_cap) stk(tr.sp++) = e[k];
-  if (e[0] != INT32_MIN) set_pending(tr, e[0]);
-  else pop_pending(tr);
+  tr.node = next;
+  return true;
 }
 
-// tests ONE triangle of the pending leaf; the next entry pops when the leaf is done
+// Split merge (default): trav_step cut into its two regions, each lane's sequence of
+// node visits and triangle tests unchanged.  trav_node visits tr.node: box
+// tests, queues the hit leaf children (child 0 first) for trav_leaf, picks
+// the next node exactly as trav_step (node = -1 when the stack is empty).
+// trav_leaf tests ONE queued triangle.  Returns: a leaf triangle is pending
+// (na > 0), else a node is pending (node >= 0), else the traversal is done.
+__device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats& st) {
+  const PtNode N = load_node(a.nodes, tr.node);
+  ++st.nodes;
+  float tn0, tn1;
+  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0);
+  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1);
+  const bool l0 = h0 && N.cnt0 > 0, l1 = h1 && N.cnt1 > 0;
+  tr.la = l0 ? N.ref0 : N.ref1;
+  tr.na = l0 ? (uint32_t)N.cnt0 : (l1 ? (uint32_t)N.cnt1 : 0u);
+  tr.lb = N.ref1;
+  tr.nb = (l0 && l1) ? (uint32_t)N.cnt1 : 0u;
+  const bool in0 = h0 && N.cnt0 == 0, in1 = h1 && N.cnt1 == 0;
+  int32_t next = -1;
+  if (in0 && in1) {
+    const bool first0 = tn0 <= tn1;
+    next = first0 ? N.ref0 : N.ref1;
+    if ((uint32_t)tr.sp < a.stack_cap) stk(tr.sp++) = first0 ? N.ref1 : N.ref0;
+  } else if (in0) {
+    next = N.ref0;
+  } else if (in1) {
+    next = N.ref1;
+  }
+  if (next < 0 && tr.sp > 0) next = stk(--tr.sp);
+  tr.node = next;
+}
+
 __device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
   tri_test(load_tri(a.tris, tr.la), tr.la, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
   ++st.tests;
   ++tr.la;
-  if (--tr.na == 0u) pop_pending(tr);
-}
-
-// one pending entry (a node visit, or a whole leaf); false when the traversal is done
-__device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
-  if (tr.node >= 0) {
-    trav_node(a, tr, o, st);
-  } else {
-    const uint32_t n = tr.na;
-    for (uint32_t k = 0; k < n; ++k) trav_leaf(a, tr, o, d, st);
+  if (--tr.na == 0u) {
+    tr.la = tr.lb;
+    tr.na = tr.nb;
+    tr.nb = 0u;
   }
-  return tr.node >= 0 || tr.na > 0u;
 }
 
 __device__ __forceinline__ int64_t closest_hit(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {

