@@ -529,22 +529,30 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
     # both kernels get the same prolog.  V = run-ahead iterations per advance round
     # (V = 1: the paper's one vote per iteration; V = 8 the default).  T = 16 is the
     # config's threshold; T = 32 = wait for every lane (Fig. 1(b)).
-    runs = (("pdom", sr.PDOM, 0, 1, 0), ("spec_t16", sr.SPEC_LOOP, 16, c.advance_unroll, 0),
-            ("spec_t16_v1", sr.SPEC_LOOP, 16, 1, 0), ("spec_t8", sr.SPEC_LOOP, 8, c.advance_unroll, 0),
-            ("spec_t32", sr.SPEC_LOOP, 32, c.advance_unroll, 0),
-            ("pdom_batch", sr.PDOM, 0, 1, 64),
-            ("spec_t16_batch", sr.SPEC_LOOP, 16, c.advance_unroll, 64),
-            ("spec_t16_v1_batch", sr.SPEC_LOOP, 16, 1, 64),
-            ("spec_t8_batch", sr.SPEC_LOOP, 8, c.advance_unroll, 64),
-            ("spec_t32_batch", sr.SPEC_LOOP, 32, c.advance_unroll, 64))
-    for name, mode, thr, V, batch in runs:
-        w = sr.divloop_workload(c.p_u32, c.fma_count, advance=V, batch=batch)
+    # "pool": Loop Merge of the Expensive() calls over a warp task pool after the
+    # batched prologs (SR_F_POOL; pool_split warps per 32 threads) -- beyond the paper's
+    # Iteration Delay, which keeps each thread's calls on its own lane
+    runs = (("pdom", sr.PDOM, 0, 1, 0, 0, 0), ("spec_t16", sr.SPEC_LOOP, 16, c.advance_unroll, 0, 0, 0),
+            ("spec_t16_v1", sr.SPEC_LOOP, 16, 1, 0, 0, 0),
+            ("spec_t8", sr.SPEC_LOOP, 8, c.advance_unroll, 0, 0, 0),
+            ("spec_t32", sr.SPEC_LOOP, 32, c.advance_unroll, 0, 0, 0),
+            ("pdom_batch", sr.PDOM, 0, 1, 64, 0, 0),
+            ("spec_t16_batch", sr.SPEC_LOOP, 16, c.advance_unroll, 64, 0, 0),
+            ("spec_t16_v1_batch", sr.SPEC_LOOP, 16, 1, 64, 0, 0),
+            ("spec_t8_batch", sr.SPEC_LOOP, 8, c.advance_unroll, 64, 0, 0),
+            ("spec_t32_batch", sr.SPEC_LOOP, 32, c.advance_unroll, 64, 0, 0),
+            ("pool", sr.SPEC_LOOP, 16, c.advance_unroll, 64, sr.F_POOL, 1),
+            (f"pool_split{c.pool_split}", sr.SPEC_LOOP, 16, c.advance_unroll, 64, sr.F_POOL,
+             c.pool_split))
+    for name, mode, thr, V, batch, fl, split in runs:
+        w = sr.divloop_workload(c.p_u32, c.fma_count, advance=V, batch=batch, flags=fl, split=split)
         t = graph_time(w, c.n_threads, c.iters, mode, thr)
         sr.sr_run(w, c.n_threads, c.iters, I.PRIMARY_SEED, mode, thr)
         exp_calls = int(ctx.region(w, c.n_threads, sr.T_COUNTERS, torch.int64)[0].item())
         res[name] = {"value": n_units / (t * 1e-3), "unit": "thread-iterations/s", "ms": t,
-                     "advance_unroll": V, "prolog_batch": batch,
+                     "advance_unroll": V, "prolog_batch": batch, "pool_split": split if fl else None,
                      "fma_frac_of_peak": exp_calls * c.fma_count / (t * 1e-3) / fma_peak}
+    res["speedup_pool_vs_pdom"] = res[f"pool_split{c.pool_split}"]["value"] / res["pdom"]["value"]
     for k in ("t16", "t16_v1", "t8", "t32"):
         res[f"speedup_{k}_vs_pdom"] = res[f"spec_{k}"]["value"] / res["pdom"]["value"]
         res[f"speedup_{k}_batch_vs_pdom_batch"] = (res[f"spec_{k}_batch"]["value"] /

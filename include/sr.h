@@ -86,6 +86,13 @@ typedef enum {
                            advance round the lanes that must shade a hit are grouped by material
                            kind (__match_any_sync); only the largest group shades, the others
                            wait for a later advance round.  Results and counters are identical. */
+#define SR_F_POOL 32u   /* DIVLOOP + SR_SPEC_LOOP (needs prolog_batch = 64): Loop Merge of the
+                           Expensive() calls over a warp task pool -- after each lane has run
+                           ahead through a window's prologs, the warp's wanted (thread,
+                           iteration) pairs are one queue and every release runs 32 of them,
+                           any lane running any thread's call; results are added to each
+                           thread's acc in iteration order.  `threshold` is not used.
+                           Results are identical. */
 
 #define SR_MAX_LAYERS 8
 typedef struct { float n, mua, mus, g, d; } sr_layer;  /* -, 1/cm, 1/cm, -, cm */
@@ -106,6 +113,11 @@ typedef struct {
                           thread; needs block_threads <= 512) (reading Q5').
                           Other values: SR_E_INVALID.  Results and schedule
                           counters are identical.                              */
+  uint32_t pool_split;   /* with SR_F_POOL: warps per group of 32 threads, each
+                          taking 64/pool_split iterations of every 64-iteration
+                          window (0 or 1 = one warp; 2; 4 -- a CTA is one group
+                          of pool_split warps, block_threads is not used).
+                          Other values: SR_E_INVALID.  Results are identical. */
 } sr_divloop_params;
 
 typedef struct {

@@ -64,13 +64,19 @@ std::string check_workload(const sr_workload* w, uint64_t n_threads) {
   if (w->block_threads > max_block(w->kind))
     return "block_threads exceeds this workload's kernels' launch bound (" +
            std::to_string(max_block(w->kind)) + ")";
-  if (w->flags & ~(SR_F_SCHED | SR_F_STATIC | SR_F_COARSE | SR_F_NOSPLIT | SR_F_MATGROUP))
+  if (w->flags & ~(SR_F_SCHED | SR_F_STATIC | SR_F_COARSE | SR_F_NOSPLIT | SR_F_MATGROUP |
+                   SR_F_POOL))
     return "unknown flags";
   switch (w->kind) {
     case SR_WL_DIVLOOP:
       if (w->divloop.fma_count % 8 != 0) return "divloop.fma_count must be a multiple of 8";
       if (w->divloop.prolog_batch > 1 && w->divloop.prolog_batch != 64)
         return "divloop.prolog_batch must be 0, 1 or 64";
+      if ((w->flags & SR_F_POOL) && w->divloop.prolog_batch != 64)
+        return "divloop: SR_F_POOL needs prolog_batch = 64";
+      if (w->divloop.pool_split > 1 &&
+          (w->divloop.pool_split != 2 && w->divloop.pool_split != 4))
+        return "divloop.pool_split must be 0, 1, 2 or 4";
       if (w->divloop.prolog_batch == 64 && w->block_threads > 512)
         return "divloop.prolog_batch = 64 needs block_threads <= 512 (64 shared-memory floats "
                "per thread)";

@@ -23,6 +23,7 @@ class DivLoop:
     fma_count: int = 1000       # Expensive() = 1000 FMAs
     threshold: int = 16
     advance_unroll: int = 8     # iterations a run-ahead lane may take per round, tuned on B200
+    pool_split: int = 4         # warp task pool (SR_F_POOL): warps per 32 threads, tuned on B200
 
 
 @dataclass(frozen=True)

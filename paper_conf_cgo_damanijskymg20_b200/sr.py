@@ -18,7 +18,7 @@ LIB_PATH = os.path.join(HERE, "libsr.so")
 SR_OK, SR_E_INVALID, SR_E_STATE, SR_E_NOMEM, SR_E_CUDA = 0, -1, -2, -3, -4
 PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
 WL_DIVLOOP, WL_COMMONCALL, WL_MCML, WL_PATHTRACE, WL_RSBENCH = 0, 1, 2, 3, 4
-F_SCHED, F_STATIC, F_COARSE, F_NOSPLIT, F_MATGROUP = 1, 2, 4, 8, 16
+F_SCHED, F_STATIC, F_COARSE, F_NOSPLIT, F_MATGROUP, F_POOL = 1, 2, 4, 8, 16, 32
 T_PERTHREAD, T_GRID, T_COUNTERS, T_SCHED, T_SCRATCH = 0, 1, 2, 3, 4
 MAX_LAYERS = 8
 N_COUNTERS = 16
@@ -46,7 +46,7 @@ class Layer(C.Structure):
 
 class DivloopParams(C.Structure):
     _fields_ = [("p_u32", C.c_uint32), ("fma_count", C.c_uint32), ("advance_unroll", C.c_uint32),
-                ("prolog_batch", C.c_uint32)]
+                ("prolog_batch", C.c_uint32), ("pool_split", C.c_uint32)]
 
 
 class CommoncallParams(C.Structure):
@@ -208,9 +208,9 @@ def scene_image_host(tris, mat, mats, cam):
 
 # ------------------------------------------------------------------ workload builders
 def divloop_workload(p_u32=1 << 29, fma_count=1000, task_offset=0, flags=0, block=0,
-                     advance=0, batch=0) -> Workload:
+                     advance=0, batch=0, split=0) -> Workload:
     w = Workload(kind=WL_DIVLOOP, flags=flags, task_offset=task_offset, block_threads=block)
-    w.divloop = DivloopParams(p_u32, fma_count, advance, batch)
+    w.divloop = DivloopParams(p_u32, fma_count, advance, batch, split)
     return w
 
 

@@ -99,6 +99,9 @@ def test_run_validation_before_state():
             sr.sr_run(bad, 64, 1, 1, sr.PDOM, 0)
         assert e.value.code == sr.SR_E_INVALID and "prolog_batch" in str(e.value)
     with pytest.raises(sr.SRError) as e:
+        sr.sr_run(sr.divloop_workload(flags=sr.F_POOL), 64, 1, 1, sr.SPEC_LOOP, 16)
+    assert e.value.code == sr.SR_E_INVALID and "SR_F_POOL" in str(e.value)
+    with pytest.raises(sr.SRError) as e:
         sr.sr_run(sr.divloop_workload(batch=64, block=1024), 64, 1, 1, sr.PDOM, 0)
     assert e.value.code == sr.SR_E_INVALID and "block_threads <= 512" in str(e.value)
 

@@ -311,6 +311,54 @@ def test_divloop_batch_schedule_matches_simulator(ctx, mode, T, V):
             assert g[0] == s["rounds"] and (g[3], g[4]) == s["ADVANCE"], wi
 
 
+# warp task pool of the Expensive() calls (SR_F_POOL, prolog_batch = 64)
+@pytest.mark.parametrize("n,iters,off,block", [(1000, 64, 0, 64), (333, 200, 0, 96), (65, 63, 0, 32),
+                                               (100, 0, 0, 64), (1, 129, 0, 64),
+                                               (97, 65, (1 << 40) + 7, 512), (32768, 64, 0, 64)])
+@pytest.mark.parametrize("split", [1, 2, 4])
+def test_divloop_pool_bit_exact(ctx, n, iters, off, block, split):
+    acc_o, cnt_o = oracle.divloop(off, n, iters, 7)
+    w = sr.divloop_workload(task_offset=off, block=block, batch=64, flags=sr.F_POOL, split=split)
+    acc, cnt, tot = run_divloop(ctx, w, n, iters, 7, sr.SPEC_LOOP, 16)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(cnt, cnt_o)
+    assert tot[0] == cnt_o.sum()
+
+
+@pytest.mark.parametrize("kw", [dict(p_u32=0), dict(p_u32=0xFFFFFFFF), dict(fma_count=8),
+                                dict(fma_count=2000)])
+@pytest.mark.parametrize("split", [1, 4])
+def test_divloop_pool_edge_cases(ctx, kw, split):
+    p = dict(p_u32=1 << 29, fma_count=1000); p.update(kw)
+    acc_o, cnt_o = oracle.divloop(0, 100, 70, 7, p["p_u32"], p["fma_count"])
+    w = sr.divloop_workload(batch=64, flags=sr.F_POOL, split=split, **kw)
+    acc, cnt, _ = run_divloop(ctx, w, 100, 70, 7, sr.SPEC_LOOP, 32)
+    assert np.array_equal(acc.view(np.uint32), acc_o.view(np.uint32))
+    assert np.array_equal(cnt, cnt_o)
+
+
+@pytest.mark.parametrize("n,iters", [(2000, 64), (77, 130)])
+@pytest.mark.parametrize("split", [1, 2, 4])
+def test_divloop_pool_schedule_closed_form(ctx, n, iters, split):
+    """per window and slice (64 / split iterations): one batched advance of every
+    valid lane, then ceil(N/32) releases running the slice's N wanted calls"""
+    w = sr.divloop_workload(flags=sr.F_SCHED | sr.F_POOL, block=64, batch=64, split=split)
+    run_divloop(ctx, w, n, iters, I.PRIMARY_SEED, sr.SPEC_LOOP, 16)
+    sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    want = oracle.divloop_wants(0, n, iters, I.PRIMARY_SEED)
+    L = 64 // split
+    for wi in range((n + 31) // 32):
+        ww = want[32 * wi:32 * wi + 32]
+        nv = len(ww)
+        Ns = [int(ww[:, b + s * L:min(b + (s + 1) * L, b + 64, iters)].sum())
+              for b in range(0, iters, 64) for s in range(split)]
+        rel = sum((N + 31) // 32 for N in Ns)
+        g = sched[wi]
+        assert g[1] == rel and g[2] == sum(Ns), wi
+        assert g[3] == len(Ns) and g[4] == len(Ns) * nv, wi
+        assert g[0] == rel + len(Ns), wi
+
+
 # ------------------------------------------------------------------ config 2
 def run_cc(ctx, w, n, iters, seed, mode):
     ctx.ensure(sr.sr_workspace_bytes(w, n))

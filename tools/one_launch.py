@@ -27,6 +27,8 @@ ap.add_argument("--pt-flags", type=int, default=0, help="extra PATHTRACE flags (
 ap.add_argument("--dl-batch", type=int, default=0, help="divloop prolog_batch (0 or 64)")
 ap.add_argument("--dl-threads", type=int, default=0, help="divloop threads (default configs[0])")
 ap.add_argument("--dl-fma", type=int, default=-1, help="divloop FMAs per Expensive (default configs[0])")
+ap.add_argument("--dl-flags", type=int, default=0, help="divloop flags (F_POOL = 32)")
+ap.add_argument("--dl-split", type=int, default=0, help="divloop pool_split")
 ap.add_argument("--rs-flags", type=int, default=0, help="extra RSBENCH flags (F_STATIC = 2)")
 a = ap.parse_args()
 modes = a.modes.split(",")
@@ -36,7 +38,8 @@ if "divloop" in a.what:
     c = I.C1
     nth = a.dl_threads or c.n_threads
     w = sr.divloop_workload(c.p_u32, c.fma_count if a.dl_fma < 0 else a.dl_fma,
-                            advance=c.advance_unroll, batch=a.dl_batch)
+                            advance=c.advance_unroll, batch=a.dl_batch, flags=a.dl_flags,
+                            split=a.dl_split)
     ctx.ensure(sr.sr_workspace_bytes(w, nth))
     for md in modes:
         sr.sr_run(w, nth, c.iters, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,

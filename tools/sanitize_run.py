@@ -41,6 +41,11 @@ if "divloop" in what:
                 run(w, 1000, iters, sr.PDOM, 0)
                 for T in (1, 16, 32):
                     run(w, 1000, iters, sr.SPEC_LOOP, T)
+                if batch:
+                    for split in (1, 2, 4):
+                        wp = sr.divloop_workload(c.p_u32, 64, advance=adv, flags=flags | sr.F_POOL,
+                                                 batch=batch, split=split)
+                        run(wp, 1000, iters, sr.SPEC_LOOP, 16)
     # one block of 1024 threads with n = 1 (31 whole warps past n)
     run(sr.divloop_workload(c.p_u32, 64, flags=sr.F_SCHED, block=1024), 1, 16, sr.SPEC_LOOP, 16)
 if "commoncall" in what:

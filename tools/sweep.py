@@ -30,6 +30,7 @@ ap.add_argument("--static", action="store_true", help="MCML static photon assign
 ap.add_argument("--iters", type=int, default=0, help="MCML photons per lane (default configs[2])")
 ap.add_argument("--prolog", type=int, default=0, help="RSBench prolog FMAs (expensive task fetch)")
 ap.add_argument("--batch", type=int, default=0, help="divloop prolog_batch (0 or 64)")
+ap.add_argument("--split", type=int, default=0, help="divloop pool_split (with --flags 32)")
 ap.add_argument("--unrolls", default="", help="comma list: sweep the merge unroll too")
 a = ap.parse_args()
 Ts = [int(x) for x in a.thresholds.split(",")]
@@ -92,7 +93,7 @@ if "divloop" in a.what:
     res = []
     for b in blocks:
         w = sr.divloop_workload(c.p_u32, c.fma_count, block=b, advance=a.unroll, batch=a.batch,
-                                flags=a.flags)
+                                flags=a.flags, split=a.split)
         ctx.ensure(sr.sr_workspace_bytes(w, c.n_threads))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
             def run():
