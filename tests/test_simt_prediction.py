@@ -14,6 +14,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, os.path.join(ROOT, "tools"))
 
 CASES = ["divloop_pdom", "divloop_spec(T=16)", "divloop_pdom_batch", "divloop_spec_batch(T=16)",
+         "divloop_pool(T=16)", "divloop_pool_split4(T=16)",
          "commoncall_pdom", "commoncall_spec",
          "rs_pdom", "rs_spec(T=32)", "rs_spec_static(T=32)",
          "mcml_pdom_static", "mcml_spec_static(T=32)", "mcml_spec_static(T=8)",

@@ -22,6 +22,8 @@ timeout 1200 ncu --metrics $M --clock-control none -k regex:"divloop|commoncall|
 # the batched-prolog divloop kernels and the static-assignment RSBench kernel
 timeout 600 ncu --metrics $M --clock-control none -k regex:divloop --csv --log-file $O/simt_dlbatch_$TAG.csv python tools/one_launch.py divloop --dl-batch 64 > /dev/null 2>&1
 timeout 600 ncu --metrics $M --clock-control none -k regex:rs_ --csv --log-file $O/simt_rsstatic_$TAG.csv python tools/one_launch.py rsbench --modes spec --rs-flags 2 > /dev/null 2>&1
+timeout 600 ncu --metrics $M --clock-control none -k regex:divloop --csv --log-file $O/simt_dlpool_$TAG.csv python tools/one_launch.py divloop --dl-batch 64 --dl-flags 32 --modes spec > /dev/null 2>&1
+timeout 600 ncu --metrics $M --clock-control none -k regex:divloop --csv --log-file $O/simt_dlpool4_$TAG.csv python tools/one_launch.py divloop --dl-batch 64 --dl-flags 32 --dl-split 4 --modes spec > /dev/null 2>&1
 # the simulator validation launches (static assignment, the oracle replays every warp)
 timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes pdom,spec --threshold 32 --unroll 1 > /dev/null 2>&1
 timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic8_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes spec --threshold 8 --unroll 1 > /dev/null 2>&1

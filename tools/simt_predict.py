@@ -76,6 +76,38 @@ def divloop_warps(mode, T, V=None, batch=False):
         yield s, len(ww)
 
 
+def divloop_pool_warps(split=1):
+    """the SR_F_POOL kernels: per window and slice (64 / split iterations) of a
+    group of 32 threads, one warp runs the slice's prologs (MASKGRP, 8 draws per
+    group) and ceil(N/32) releases of its N wanted calls (STEP: N lanes in all);
+    warp 0 then adds every thread's results in order (EPIK: as many trips as the
+    thread with the most calls, one lane per call).  Closed-form counts."""
+    c = I.C1
+    want = oracle.divloop_wants(0, c.n_threads, c.iters, I.PRIMARY_SEED, c.p_u32)
+    L = 64 // split
+    for w in range(0, c.n_threads, 32):
+        ww = want[w:w + 32].astype(np.int64)
+        nv = len(ww)
+        for sl in range(split):
+            rel = lanes = groups = 0
+            epik_x = epik_l = 0
+            for b in range(0, c.iters, 64):
+                lo, hi = b + sl * L, min(b + (sl + 1) * L, b + 64, c.iters)
+                cnt = ww[:, lo:hi].sum(1) if hi > lo else np.zeros(nv, np.int64)
+                N = int(cnt.sum())
+                rel += (N + 31) // 32
+                lanes += N
+                groups += (max(hi - lo, 0) + 7) // 8
+                if sl == 0:   # warp 0 adds every slice's results
+                    for s2 in range(split):
+                        l2, h2 = b + s2 * L, min(b + (s2 + 1) * L, b + 64, c.iters)
+                        c2 = ww[:, l2:h2].sum(1) if h2 > l2 else np.zeros(nv, np.int64)
+                        epik_x += int(c2.max()) if nv else 0
+                        epik_l += int(c2.sum())
+            yield {"MASKGRP": (groups, groups * nv), "RELEASE": (rel, 32 * rel),
+                   "STEP": (rel, lanes), "EPIK": (epik_x, epik_l), "rounds": rel}, nv
+
+
 def commoncall_warps(mode):
     c = I.C2
     _, arm = oracle.commoncall(0, c.n_threads, 1, I.PRIMARY_SEED, c.split_u32, fma_count=0)
@@ -156,6 +188,9 @@ CASES = {
                            lambda: divloop_warps(oracle.PDOM, 0, batch=True)),
     "divloop_spec_batch(T=16)": (r"divloop_spec_batchILi125ELb0",
                                  lambda: divloop_warps(oracle.SPEC_LOOP, 16, batch=True)),
+    "divloop_pool(T=16)": (r"divloop_poolILi125ELb0", lambda: divloop_pool_warps(1)),
+    "divloop_pool_split4(T=16)": (r"divloop_pool_splitILi125ELb0ELi4",
+                                  lambda: divloop_pool_warps(4)),
     "mcml_pdom": (r"mcml_pdomILb1ELb0ELb1", lambda: mcml_dyn_warps(oracle.PDOM, 0)),
     "mcml_spec(T=32)": (r"mcml_specILb1ELb0ELb1", lambda: mcml_dyn_warps(oracle.SPEC_LOOP, 32)),
 }

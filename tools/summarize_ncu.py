@@ -29,6 +29,8 @@ LABELS_ALL = ["divloop_pdom", "divloop_spec(T=16)", "commoncall_pdom", "commonca
               f"pt_spec(T={_I.C4.threshold})"]
 LABELS_DLBATCH = ["divloop_pdom_batch", "divloop_spec_batch(T=16)"]
 LABELS_RSSTATIC = [f"rs_spec_static(T={_TRS})"]
+LABELS_DLPOOL = ["divloop_pool(T=16)"]
+LABELS_DLPOOL4 = ["divloop_pool_split4(T=16)"]
 LABELS_MCSTATIC = ["mcml_pdom_static", "mcml_spec_static(T=32)"]
 LABELS_MCSTATIC8 = ["mcml_spec_static(T=8)"]
 LABELS_MCSTATICU4 = ["mcml_spec_static(T=32,U=4)"]
@@ -106,7 +108,9 @@ def main():
                           (f"simt_mcstatic8_{tag}.csv", LABELS_MCSTATIC8),
                           (f"simt_mcstaticu4_{tag}.csv", LABELS_MCSTATICU4),
                           (f"simt_dlbatch_{tag}.csv", LABELS_DLBATCH),
-                          (f"simt_rsstatic_{tag}.csv", LABELS_RSSTATIC)):
+                          (f"simt_rsstatic_{tag}.csv", LABELS_RSSTATIC),
+                          (f"simt_dlpool_{tag}.csv", LABELS_DLPOOL),
+                          (f"simt_dlpool4_{tag}.csv", LABELS_DLPOOL4)):
         path = os.path.join(OUT, fname)
         if not os.path.exists(path):
             continue
