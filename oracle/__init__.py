@@ -20,7 +20,7 @@ import numpy as np
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB = os.path.join(HERE, "liboracle.so")
 SOURCES = ["philox.c", "srmath.c", "divloop.c", "commoncall.c", "mcml.c", "warpsim.c",
-           "pathtrace.c", "rsbench.c"]
+           "pathtrace.c", "rsbench.c", "pttrace.c"]
 CFLAGS = ["-O2", "-std=gnu11", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared",
           "-Wall", "-Wno-unused-function"]
 
@@ -29,6 +29,10 @@ PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
 # region ids (oracle.h)
 DL = dict(ENTRY=0, PROLOG=1, EXPENSIVE=2, EPILOG=3, ROUND=4, RELEASE=5, ADVANCE=6)
 CC = dict(ENTRY=0, THEN=1, ELSE_PRE=2, CALL=3, ELSE_POST=4, MERGE=5)
+PT = {k: i for i, k in enumerate(
+    "ENTRY OUTER LAUNCH BOUNCE TBEGIN STEP NODE PUSH NOPUSH NEXTNONE POP LEAFIF LEAF TT TT_U "
+    "TT_V TT_T TT_ID TT_UPD SH SH_HIT SH_SURF SH_DIFF SH_MIRR SH_GLASS SH_RR SH_END ROUND REL "
+    "LREL NREL ADV".split())}
 LM = dict(ENTRY=0, LAUNCH=1, STEP=2, STEP_BOUNDARY=3, STEP_INTERACT=4, ROUND=5, RELEASE=6,
           ADVANCE=7, **{f"EV{b}": 8 + b for b in range(16)}, **{f"NEV{b}": 24 + b for b in range(16)},
           A_RR=40, B_RR=41, B_REL=42, BI=43, A_TAIL=44, CLAIM=45, CLAIMIT=46, CHUNK=47)
@@ -302,6 +306,44 @@ def ws_loopmerge_raw(nsteps, ev_flat, ev_off, mode, T, W=32, U=1):
                             None if ev_off is None else _p(ev_off, C.c_uint64),
                             W, n_valid, K, mode, T, U, C.byref(o))
     return o.as_dict(LM)
+
+
+def pt_trace(img, width, height, spp, max_depth, seed, pixels=None, cap=None):
+    """(ops uint16, off uint64[n+1], rgb float32[n, 3]) -- see oracle.h or_pt_trace.
+    img: the scene image (uint8 numpy array, sr_scene_build_host)."""
+    img = np.ascontiguousarray(img, np.uint8)
+    n = width * height if pixels is None else len(pixels)
+    pix = None if pixels is None else np.ascontiguousarray(pixels, np.uint32)
+    cap = cap or n * spp * 400
+    L = lib()
+    L.or_pt_trace.argtypes = [C.POINTER(C.c_uint8), C.c_uint64, C.c_uint32, C.c_uint32,
+                              C.c_uint32, C.c_uint32, C.c_uint64, C.POINTER(C.c_uint32),
+                              C.c_uint32, C.POINTER(C.c_uint16), C.c_uint64,
+                              C.POINTER(C.c_uint64), C.POINTER(C.c_float)]
+    L.or_pt_trace.restype = C.c_uint64
+    ops = np.zeros(cap, np.uint16)
+    off = np.zeros(n + 1, np.uint64)
+    rgb = np.zeros((n, 3), np.float32)
+    used = L.or_pt_trace(_p(img, C.c_uint8), img.size, width, height, spp, max_depth, seed,
+                         None if pix is None else _p(pix, C.c_uint32), n, _p(ops, C.c_uint16),
+                         cap, _p(off, C.c_uint64), _p(rgb, C.c_float))
+    if used == 2**64 - 2:
+        raise ValueError("not a scene image")
+    if used == 2**64 - 1:
+        return pt_trace(img, width, height, spp, max_depth, seed, pixels, cap * 4)
+    return ops[:used], off, rgb
+
+
+def ws_pt(ops, off, mode, T=0, U=1):
+    """one warp's PDOM / split Loop Merge schedule (off: n_valid + 1 offsets)"""
+    ops = np.ascontiguousarray(ops, np.uint16)
+    off = np.ascontiguousarray(off, np.uint64)
+    o = WsCounts()
+    L = lib()
+    L.ws_pt.argtypes = [C.POINTER(C.c_uint16), C.POINTER(C.c_uint64), C.c_uint32, C.c_int,
+                        C.c_uint32, C.c_uint32, C.POINTER(WsCounts)]
+    L.ws_pt(_p(ops, C.c_uint16), _p(off, C.c_uint64), len(off) - 1, mode, T, U, C.byref(o))
+    return o.as_dict(PT)
 
 
 def ws_loopmerge_stream(nsteps, mode, T, U=1, W=32, ev=None, ev_off=None):

@@ -129,6 +129,21 @@ void or_pt_render(const or_pt_scene* sc, uint32_t width, uint32_t height, uint32
                   uint32_t max_depth, uint64_t seed, const uint32_t* pixels, uint32_t n_pixels,
                   float* rgb, uint64_t* counters);
 
+/* ---- pttrace.c : the path tracer's work-item streams and schedules (oracle
+ * part 2; see pttrace.c).  Op encoding (uint16): */
+#define OR_PT_OP_NODE 0x0000u   /* node visit: n0 | n1 << 4 | push << 8 | pop << 9 | end << 10 */
+#define OR_PT_OP_PATH 0x2000u   /* a path (sample) starts: camera ray                       */
+#define OR_PT_OP_SHADE 0x4000u  /* a ray's shading: outcome | rr << 3 | path ends << 4      */
+#define OR_PT_OP_LEAF 0x8000u   /* one triangle test: stage (0..5, see pttrace.c)           */
+enum { OR_PT_SH_MISS = 0, OR_PT_SH_LIGHT, OR_PT_SH_DIFFUSE, OR_PT_SH_MIRROR, OR_PT_SH_GLASS };
+/* rays / node visits / triangle tests of pixels[0..n_pixels) as per-lane op
+ * streams (lane k: ops[off[k] .. off[k+1])) and, if rgb != NULL, their pixel
+ * sums (must equal or_pt_render's).  Returns ops used, UINT64_MAX if cap is too
+ * small, UINT64_MAX - 1 for a bad image. */
+uint64_t or_pt_trace(const unsigned char* img, uint64_t img_bytes, uint32_t width, uint32_t height,
+                     uint32_t spp, uint32_t max_depth, uint64_t seed, const uint32_t* pixels,
+                     uint32_t n_pixels, uint16_t* ops, uint64_t cap, uint64_t* off, float* rgb);
+
 /* ---- rsbench.c : NEXT-1, RSBench-shaped nested trip-count loop (Fig. 3). */
 enum { OR_TAG_RS = 5 };
 #define OR_RS_MATS 12
@@ -215,6 +230,16 @@ void ws_loopmerge(const uint32_t* nsteps, const or_event* ev, const uint64_t* ev
  * executions over ALL legal interleavings of the iteration-delay program
  * (any parked subset may be released, any free lane may advance). */
 uint32_t ws_divloop_optimum(const uint8_t* want, uint32_t W, uint32_t L);
+/* path tracer schedules (pttrace.c; ops from or_pt_trace) */
+enum { WS_PT_ENTRY = 0, WS_PT_OUTER, WS_PT_LAUNCH, WS_PT_BOUNCE, WS_PT_TBEGIN, WS_PT_STEP,
+       WS_PT_NODE, WS_PT_PUSH, WS_PT_NOPUSH, WS_PT_NEXTNONE, WS_PT_POP, WS_PT_LEAFIF,
+       WS_PT_LEAF, WS_PT_TT, WS_PT_TT_U, WS_PT_TT_V, WS_PT_TT_T, WS_PT_TT_ID, WS_PT_TT_UPD,
+       WS_PT_SH, WS_PT_SH_HIT, WS_PT_SH_SURF, WS_PT_SH_DIFF, WS_PT_SH_MIRR, WS_PT_SH_GLASS,
+       WS_PT_SH_RR, WS_PT_SH_END, WS_PT_ROUND, WS_PT_REL, WS_PT_LREL, WS_PT_NREL, WS_PT_ADV };
+/* the PDOM (mode WS_PDOM) or split Loop Merge (WS_SPEC_LOOP, threshold T, U
+ * work items per release) schedule of one warp of n_valid lanes */
+void ws_pt(const uint16_t* ops, const uint64_t* off, uint32_t n_valid, int mode, uint32_t T,
+           uint32_t U, ws_counts* out);
 
 #ifdef __cplusplus
 }

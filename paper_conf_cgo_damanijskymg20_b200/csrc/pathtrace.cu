@@ -151,29 +151,29 @@ __device__ __forceinline__ bool box_hit(const float* lo, const float* hi, V3 o, 
 // binary32 subtractions).
 __device__ __forceinline__ void tri_test(const PtTri& T, int32_t at, V3 o, V3 d, float& tb,
                                          int32_t& ib, uint32_t& mb, uint32_t& slot) {
-  const V3 v0 = mk(T.v0[0], T.v0[1], T.v0[2]);
+  const V3 v0 = mk(T.v0[0], T.v0[1], T.v0[2]);  // @sr-region TT
   const V3 e1 = mk(T.e1[0], T.e1[1], T.e1[2]);
   const V3 e2 = mk(T.e2[0], T.e2[1], T.e2[2]);
   const V3 pv = cross(d, e2);
   const float det = dot(e1, pv);
   if (fabsf(det) < kDetEps) return;
-  const float inv = 1.0f / det;
+  const float inv = 1.0f / det;  // @sr-region TT_U
   const V3 tv = sub(o, v0);
   const float u = dot(tv, pv) * inv;
   if (u < 0.0f || u > 1.0f) return;
-  const V3 qv = cross(tv, e1);
+  const V3 qv = cross(tv, e1);  // @sr-region TT_V
   const float v = dot(d, qv) * inv;
   if (v < 0.0f || u + v > 1.0f) return;
-  const float t = dot(e2, qv) * inv;
+  const float t = dot(e2, qv) * inv;  // @sr-region TT_T
   if (!(t > kTmin)) return;
-  const int32_t id = (int32_t)T.id;        // < 2^31 (sr_scene_build checks)
+  const int32_t id = (int32_t)T.id;  // < 2^31 (sr_scene_build checks)  // @sr-region TT_ID
   if (t < tb || (t == tb && id < ib)) {   // ties -> smaller original id (= brute force)
-    tb = t;
+    tb = t;  // @sr-region TT_UPD
     ib = id;
     mb = T.mat;
     slot = (uint32_t)at;
   }
-}
+}  // @sr-region END
 
 // Resumable BVH traversal: one call of trav_step visits one node (its two
 // child boxes, the triangles of child leaves, push/pop).  closest_hit() runs
@@ -218,42 +218,37 @@ __device__ __forceinline__ void trav_begin(Trav& tr, V3 d) {
 
 // returns false when the traversal is finished
 __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
-  const PtNode N = load_node(a.nodes, tr.node);
+  const PtNode N = load_node(a.nodes, tr.node);  // @sr-region NODE
   ++st.nodes;
   float tn0, tn1;
   const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0);
   const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1);
-  // leaves: test their triangles now; inner children: descend / push
-  if (h0 && N.cnt0 > 0) {
-    for (int32_t k = 0; k < N.cnt0; ++k) {
-      tri_test(load_tri(a.tris, N.ref0 + k), N.ref0 + k, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
-      ++st.tests;
-    }
+  // leaves: test their triangles now (child 0's, then child 1's, one loop);
+  // inner children: descend / push
+  const int32_t n0 = (h0 && N.cnt0 > 0) ? N.cnt0 : 0, n1 = (h1 && N.cnt1 > 0) ? N.cnt1 : 0;
+  for (int32_t k = 0; k < n0 + n1; ++k) {  // @sr-region LEAFIF
+    const int32_t at = k < n0 ? N.ref0 + k : N.ref1 + (k - n0);  // @sr-region LEAF
+    tri_test(load_tri(a.tris, at), at, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
+    ++st.tests;
   }
-  if (h1 && N.cnt1 > 0) {
-    for (int32_t k = 0; k < N.cnt1; ++k) {
-      tri_test(load_tri(a.tris, N.ref1 + k), N.ref1 + k, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
-      ++st.tests;
-    }
-  }
-  const bool in0 = h0 && N.cnt0 == 0, in1 = h1 && N.cnt1 == 0;
+  const bool in0 = h0 && N.cnt0 == 0, in1 = h1 && N.cnt1 == 0;  // @sr-region NODE
   int32_t next = -1;
   if (in0 && in1) {
-    const bool first0 = tn0 <= tn1;
+    const bool first0 = tn0 <= tn1;  // @sr-region PUSH
     next = first0 ? N.ref0 : N.ref1;
     if ((uint32_t)tr.sp < a.stack_cap) stk(tr.sp++) = first0 ? N.ref1 : N.ref0;
   } else if (in0) {
-    next = N.ref0;
+    next = N.ref0;  // @sr-region NOPUSH
   } else if (in1) {
     next = N.ref1;
   }
-  if (next < 0) {
-    if (tr.sp == 0) return false;
-    next = stk(--tr.sp);
+  if (next < 0) {  // @sr-region NODE
+    if (tr.sp == 0) return false;  // @sr-region NEXTNONE
+    next = stk(--tr.sp);  // @sr-region POP
   }
-  tr.node = next;
+  tr.node = next;  // @sr-region NODE
   return true;
-}
+}  // @sr-region END
 
 // Split merge (default): trav_step cut into its two regions, each lane's sequence of
 // node visits and triangle tests unchanged.  trav_node visits tr.node: box
@@ -262,7 +257,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d,
 // trav_leaf tests ONE queued triangle.  Returns: a leaf triangle is pending
 // (na > 0), else a node is pending (node >= 0), else the traversal is done.
 __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats& st) {
-  const PtNode N = load_node(a.nodes, tr.node);
+  const PtNode N = load_node(a.nodes, tr.node);  // @sr-region NODE
   ++st.nodes;
   float tn0, tn1;
   const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0);
@@ -275,20 +270,22 @@ __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats
   const bool in0 = h0 && N.cnt0 == 0, in1 = h1 && N.cnt1 == 0;
   int32_t next = -1;
   if (in0 && in1) {
-    const bool first0 = tn0 <= tn1;
+    const bool first0 = tn0 <= tn1;  // @sr-region PUSH
     next = first0 ? N.ref0 : N.ref1;
     if ((uint32_t)tr.sp < a.stack_cap) stk(tr.sp++) = first0 ? N.ref1 : N.ref0;
   } else if (in0) {
-    next = N.ref0;
+    next = N.ref0;  // @sr-region NOPUSH
   } else if (in1) {
     next = N.ref1;
   }
-  if (next < 0 && tr.sp > 0) next = stk(--tr.sp);
-  tr.node = next;
-}
+  if (next < 0) {  // @sr-region NODE
+    if (tr.sp > 0) next = stk(--tr.sp);  // @sr-region POP
+  }
+  tr.node = next;  // @sr-region NODE
+}  // @sr-region END
 
 __device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
-  tri_test(load_tri(a.tris, tr.la), tr.la, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
+  tri_test(load_tri(a.tris, tr.la), tr.la, o, d, tr.tb, tr.ib, tr.mb, tr.slot);  // @sr-region LEAF
   ++st.tests;
   ++tr.la;
   if (--tr.na == 0u) {
@@ -296,14 +293,14 @@ __device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, V3 o, V3 d,
     tr.na = tr.nb;
     tr.nb = 0u;
   }
-}
+}  // @sr-region END
 
 __device__ __forceinline__ int64_t closest_hit(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
-  trav_begin(tr, d);
-  while (trav_step(a, tr, o, d, st)) {
+  trav_begin(tr, d);  // @sr-region TBEGIN
+  while (trav_step(a, tr, o, d, st)) {  // @sr-region STEP
   }
-  return (int64_t)tr.ib;
-}
+  return (int64_t)tr.ib;  // @sr-region BOUNCE
+}  // @sr-region END
 
 struct Path {
   V3 o, d, thr, rad;   // the pixel sum lives in a.rgb (this lane's pixel only)
@@ -312,7 +309,7 @@ struct Path {
 };
 
 __device__ __forceinline__ void camera_ray(const PtArgs& a, const PtHeader& H, Path& p) {
-  const uint64_t q = (uint64_t)p.pix * a.spp + p.s;
+  const uint64_t q = (uint64_t)p.pix * a.spp + p.s;  // @sr-region LAUNCH
   const uint4 u = draw(0u, kTagPt, q, a.keys);
   const uint32_t px = p.pix % a.width, py = p.pix / a.width;
   const float fx = ((float)px + u01(u.x)) / (float)a.width;
@@ -329,7 +326,7 @@ __device__ __forceinline__ void camera_ray(const PtArgs& a, const PtHeader& H, P
   p.rad = mk(0.0f, 0.0f, 0.0f);
   p.b = 0;
   p.alive = true;
-}
+}  // @sr-region END
 
 __device__ __forceinline__ void onb(V3 n, V3& t1, V3& t2) {
   const float sign = copysignf(1.0f, n.z);
@@ -344,18 +341,18 @@ __device__ __forceinline__ void onb(V3 n, V3& t1, V3& t2) {
 // max_depth or lost the roulette; the epilog (pixel sum) happens at that
 // point, in sample order.
 __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
-  const int64_t hit = tr.ib;
+  const int64_t hit = tr.ib;  // @sr-region SH
   const float t = tr.tb;
   const uint32_t mat = tr.mb, slot = tr.slot;
   bool end = hit < 0;
   if (!end) {
-    const PtMat m = load_mat(a.mats, mat);
+    const PtMat m = load_mat(a.mats, mat);  // @sr-region SH_HIT
     const uint32_t kind = (uint32_t)m.kind;
     p.rad = add(p.rad, mk(p.thr.x * m.er, p.thr.y * m.eg, p.thr.z * m.eb));
     if (kind == 3u) {
       end = true;
     } else {
-      const PtTri T = load_tri(a.tris, (int32_t)slot);
+      const PtTri T = load_tri(a.tris, (int32_t)slot);  // @sr-region SH_SURF
       const V3 e1 = mk(T.e1[0], T.e1[1], T.e1[2]);
       const V3 e2 = mk(T.e2[0], T.e2[1], T.e2[2]);
       const V3 ng = normalize(cross(e1, e2));
@@ -366,7 +363,7 @@ __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
       const uint64_t q = (uint64_t)p.pix * a.spp + p.s;
       const uint4 u = draw(p.b + 1u, kTagPt, q, a.keys);
       if (kind == 0u) {
-        const float r1 = u01(u.x);
+        const float r1 = u01(u.x);  // @sr-region SH_DIFF
         const float rr = sqrtf(r1);
         float sp, cp;
         sr_sincos2pif(u01(u.y), sp, cp);
@@ -375,9 +372,9 @@ __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
         onb(n, t1, t2);
         p.d = add(add(scl(t1, lx), scl(t2, ly)), scl(n, lz));
       } else if (kind == 1u) {
-        p.d = sub(p.d, scl(n, 2.0f * dot(p.d, n)));
+        p.d = sub(p.d, scl(n, 2.0f * dot(p.d, n)));  // @sr-region SH_MIRR
       } else {
-        const float ior = m.ior;
+        const float ior = m.ior;  // @sr-region SH_GLASS
         const float eta = entering ? 1.0f / ior : ior;
         const float cosi = -dot(p.d, n);
         const float k = 1.0f - eta * eta * (1.0f - cosi * cosi);
@@ -388,35 +385,35 @@ __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
         if (k < 0.0f || u01(u.z) < fr) p.d = sub(p.d, scl(n, 2.0f * dot(p.d, n)));
         else p.d = add(scl(p.d, eta), scl(n, eta * cosi - sqrtf(k)));
       }
-      p.thr = mk(p.thr.x * m.r, p.thr.y * m.g, p.thr.z * m.b);
+      p.thr = mk(p.thr.x * m.r, p.thr.y * m.g, p.thr.z * m.b);  // @sr-region SH_SURF
       p.o = pt;
       if (p.b >= 3u) {
-        const float pm = fmaxf(p.thr.x, fmaxf(p.thr.y, p.thr.z));
+        const float pm = fmaxf(p.thr.x, fmaxf(p.thr.y, p.thr.z));  // @sr-region SH_RR
         const float prr = fminf(0.95f, pm);
         if (!(u01(u.w) < prr)) end = true;
         else p.thr = mk(p.thr.x / prr, p.thr.y / prr, p.thr.z / prr);
       }
     }
   }
-  p.b = p.b + 1u;
+  p.b = p.b + 1u;  // @sr-region SH
   if (!end && p.b >= a.max_depth) end = true;
   if (end) {
     // Epilog: pixel += radiance, in sample order, in the output itself (a lane owns
     // its pixel; one read-modify-write per path keeps three registers free)
-    float* px = a.rgb + 3 * (uint64_t)p.pix;
+    float* px = a.rgb + 3 * (uint64_t)p.pix;  // @sr-region SH_END
     px[0] = px[0] + p.rad.x;
     px[1] = px[1] + p.rad.y;
     px[2] = px[2] + p.rad.z;
     p.alive = false;
   }
-}
+}  // @sr-region END
 
 __device__ __forceinline__ void finish(const PtArgs& a, const Path& p, bool valid, Stats st,
                                        uint32_t paths, uint64_t warp, uint32_t rounds,
                                        uint32_t rel, uint32_t rel_lanes, uint32_t adv,
                                        uint32_t adv_lanes, uint32_t lrel = 0,
                                        uint32_t lrel_lanes = 0) {
-  unsigned long long v[4] = {paths, st.rays, st.nodes, st.tests};
+  unsigned long long v[4] = {paths, st.rays, st.nodes, st.tests};  // @sr-region ENTRY:full
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
 #pragma unroll
@@ -431,17 +428,17 @@ __device__ __forceinline__ void finish(const PtArgs& a, const Path& p, bool vali
       s[1] = make_uint4(adv_lanes, lrel, lrel_lanes, 0u);
     }
   }
-}
+}  // @sr-region END
 
 __device__ __forceinline__ void bounce(const PtArgs& a, Path& p, Trav& tr, Stats& st) {
-  closest_hit(a, tr, p.o, p.d, st);
+  closest_hit(a, tr, p.o, p.d, st);  // @sr-region BOUNCE
   ++st.rays;
   shade(a, p, tr);
-}
+}  // @sr-region END
 
 template <bool SCHED>
 __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_PDOM) pt_pdom(const PtArgs a) {
-  const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
+  const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);  // @sr-region ENTRY:full
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = g < a.n;
   Path p;
@@ -454,22 +451,22 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_PDOM) pt_pdom(const PtA
   Trav tr;
   Stats st{0, 0, 0};
   uint32_t paths = 0, outer = 0, rel = 0, rel_lanes = 0, launch_lanes = 0;
-  for (uint32_t s = 0; s < a.spp; ++s) {
+  for (uint32_t s = 0; s < a.spp; ++s) {  // @sr-region OUTER:full
     if (SCHED) { ++outer; launch_lanes += __popc(__ballot_sync(kFull, valid)); }
     if (valid) {
-      p.s = s;
+      p.s = s;  // @sr-region LAUNCH
       camera_ray(a, H, p);              // Prolog
       ++paths;
-      do {                              // L1: bounce loop, divergent trip count
+      do {                              // L1: bounce loop, divergent trip count  // @sr-region BOUNCE
         if constexpr (SCHED) {
           const uint32_t m = __activemask();
           if (lane_id() == (uint32_t)(__ffs(m) - 1)) { ++rel; rel_lanes += __popc(m); }
         }
         bounce(a, p, tr, st);
-      } while (p.alive);
-    }                                   // IPDOM: reconverge, next sample
+      } while (p.alive);  // @sr-region BOUNCE
+    }                                   // IPDOM: reconverge, next sample  // @sr-region OUTER:full
   }
-  uint32_t r = 0, rl = 0;
+  uint32_t r = 0, rl = 0;  // @sr-region ENTRY:full
   if constexpr (SCHED) { r = __reduce_add_sync(kFull, rel); rl = __reduce_add_sync(kFull, rel_lanes); }
   finish(a, p, valid, st, paths, g >> 5, outer, r, rl, outer, launch_lanes);
 }
@@ -489,7 +486,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_PDOM) pt_pdom(const PtA
 // in R for a later one.  A miss forms its own group.
 template <bool SCHED, bool NODE, bool SPLIT = false, bool MATG = false>
 __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) {
-  const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);
+  const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);  // @sr-region ENTRY:full
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = g < a.n;
   Path p;
@@ -507,7 +504,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
   uint32_t next_s = 0;
   uint32_t E = __ballot_sync(kFull, !valid || a.spp == 0);  // lanes with nothing left to do
   uint32_t lrel = 0, lrel_lanes = 0;
-  for (;;) {
+  for (;;) {  // @sr-region ROUND:full
     if constexpr (SPLIT) {
       // two concurrent predictions: I = lanes at a BVH node, L = lanes with a
       // leaf triangle pending.  Vote: the larger group G is the candidate
@@ -521,20 +518,20 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
       const uint32_t G = leaf ? L : I;
       if (G != 0u && ((uint32_t)__popc(G) >= a.T || R == 0u)) {
         if ((G >> lane_id()) & 1u) {
-          __syncwarp(G);
+          __syncwarp(G);  // @sr-region REL
           if (leaf) {
-            if constexpr (SCHED) { ++lrel; lrel_lanes += __popc(G); }
-            for (uint32_t k = 0; k < a.unroll && tr.na > 0u; ++k) trav_leaf(a, tr, p.o, p.d, st);
+            if constexpr (SCHED) { ++lrel; lrel_lanes += __popc(G); }  // @sr-region LREL
+            for (uint32_t k = 0; k < a.unroll && tr.na > 0u; ++k) trav_leaf(a, tr, p.o, p.d, st);  // @sr-region LEAF
           } else {
-            if constexpr (SCHED) { ++rel; rel_lanes += __popc(G); }
-            for (uint32_t k = 0; k < a.unroll && tr.na == 0u && tr.node >= 0; ++k)
+            if constexpr (SCHED) { ++rel; rel_lanes += __popc(G); }  // @sr-region NREL
+            for (uint32_t k = 0; k < a.unroll && tr.na == 0u && tr.node >= 0; ++k)  // @sr-region STEP
               trav_node(a, tr, p.o, st);
           }
-          trav = tr.na > 0u || tr.node >= 0;
+          trav = tr.na > 0u || tr.node >= 0;  // @sr-region REL
         }
-        continue;
+        continue;  // @sr-region ROUND:full
       }
-      if constexpr (SCHED) { ++adv; adv_lanes += __popc(R); }
+      if constexpr (SCHED) { ++adv; adv_lanes += __popc(R); }  // @sr-region ADV:full
       bool go = (R >> lane_id()) & 1u;
       if constexpr (MATG) {
         const bool needs = go && p.alive;   // a finished traversal whose hit must be shaded
@@ -549,22 +546,22 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
         }
       }
       if (go) {
-        if (p.alive) shade(a, p, tr);
+        if (p.alive) shade(a, p, tr);  // @sr-region ADV
         if (!p.alive && next_s < a.spp) {
-          p.s = next_s++;
+          p.s = next_s++;  // @sr-region LAUNCH
           camera_ray(a, H, p);
           ++paths;
         }
-        if (p.alive) {
-          trav_begin(tr, p.d);
+        if (p.alive) {  // @sr-region ADV
+          trav_begin(tr, p.d);  // @sr-region TBEGIN
           ++st.rays;
           trav = true;
         }
       }
-      E = __ballot_sync(kFull, !valid || (!p.alive && next_s >= a.spp));
+      E = __ballot_sync(kFull, !valid || (!p.alive && next_s >= a.spp));  // @sr-region ADV:full
       continue;
     }
-    const uint32_t P = __ballot_sync(kFull, NODE ? trav : p.alive);
+    const uint32_t P = __ballot_sync(kFull, NODE ? trav : p.alive);  // @sr-region ROUND:full
     const uint32_t R = ~(P | E);
     if ((P | R) == 0u) break;
     if constexpr (SCHED) ++rounds;
@@ -595,7 +592,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
       E = __ballot_sync(kFull, !valid || (!p.alive && next_s >= a.spp));
     }
   }
-  finish(a, p, valid, st, paths, g >> 5, rounds, rel, rel_lanes, adv, adv_lanes, lrel,
+  finish(a, p, valid, st, paths, g >> 5, rounds, rel, rel_lanes, adv, adv_lanes, lrel,  // @sr-region ENTRY:full
          lrel_lanes);
 }
 

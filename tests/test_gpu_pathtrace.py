@@ -110,3 +110,37 @@ def test_render_full_config_invariants_and_sampled_pixels(ctx):
     ref, _ = oracle.pt_render(oracle.pt_scene(tris, mat, mats, cam), cfg.width, cfg.height,
                               cfg.spp, cfg.max_depth, I.PRIMARY_SEED, pixels=pix)
     assert np.array_equal(a[pix].view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("mode,T", [(sr.PDOM, 0), (sr.SPEC_LOOP, 12), (sr.SPEC_LOOP, 32),
+                                    (sr.SPEC_LOOP, 1)])
+def test_schedule_matches_simulator(ctx, mode, T):
+    """per-warp schedule counters of the instrumented kernels (split merge, U = 8)
+    == the path-tracer warp simulator replaying the oracle's work-item streams"""
+    cfg = I.C4_SMALL
+    tris, mat, mats, cam, buf, used = scene(cfg)
+    n = cfg.width * cfg.height
+    w = sr.pathtrace_workload(buf.data_ptr(), used, cfg.width, cfg.height, cfg.max_depth,
+                              flags=sr.F_SCHED)
+    ctx.ensure(sr.sr_workspace_bytes(w, n))
+    sr.sr_run(w, n, cfg.spp, I.PRIMARY_SEED, mode, T)
+    sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
+    cnt = ctx.region(w, n, sr.T_COUNTERS, torch.int64).cpu().numpy()
+    img = sr.scene_image_host(tris, mat, mats, cam)
+    ops, off, _ = oracle.pt_trace(img, cfg.width, cfg.height, cfg.spp, cfg.max_depth,
+                                  I.PRIMARY_SEED)
+    node = (ops & 0xE000) == 0
+    leaf = (ops & 0x8000) != 0
+    assert cnt[2] == int(node.sum()) and cnt[3] == int(leaf.sum())   # node visits, tests
+    for wi in range(n // 32):
+        o = off[32 * wi:32 * wi + 33]
+        s = oracle.ws_pt(ops[o[0]:o[-1]], o - o[0],
+                         oracle.PDOM if mode == sr.PDOM else oracle.SPEC_LOOP, T, 8)
+        g = sched[wi]
+        if mode == sr.PDOM:
+            assert (g[1], g[2]) == s["BOUNCE"], wi
+            assert g[0] == s["OUTER"][0] and g[4] == s["LAUNCH"][1], wi
+        else:
+            assert g[0] == s["rounds"], wi
+            assert (g[1], g[2]) == s["NREL"] and (g[5], g[6]) == s["LREL"], wi
+            assert (g[3], g[4]) == s["ADV"], wi

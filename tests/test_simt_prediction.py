@@ -20,7 +20,9 @@ CASES = ["divloop_pdom", "divloop_spec(T=16)", "divloop_pdom_batch", "divloop_sp
          "mcml_pdom_static", "mcml_spec_static(T=32)", "mcml_spec_static(T=8)",
          "mcml_spec_static(T=32,U=4)",
          # the bench's own launches: dynamic photon claiming, U = 4 (sampled warps)
-         "mcml_pdom", "mcml_spec(T=32)"]
+         "mcml_pdom", "mcml_spec(T=32)",
+         # configs[3]: the path tracer (sampled warps; oracle.pt_trace work-item streams)
+         "pt_pdom", "pt_spec(T=12)"]
 
 
 @pytest.fixture(scope="module")
@@ -30,8 +32,8 @@ def prediction():
     import sass_regions
     import simt_predict
     measured = json.load(open(os.path.join(ROOT, "profiles", "simt_efficiency.json")))
-    hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_|rs_")
-    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_|rs_")
+    hashes = sass_regions.kernel_hashes("divloop_|commoncall_|mcml_|rs_|pt_")
+    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_|rs_|pt_")
     return measured, hashes, costs, simt_predict
 
 

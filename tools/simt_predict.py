@@ -145,6 +145,36 @@ def rsbench_warps(mode, T, U=None, pool=False):
             yield oracle.ws_loopmerge(tr, mode, T, U=U if mode == oracle.SPEC_LOOP else 1), len(tr)
 
 
+# configs[3]: the path tracer's warps are 32 consecutive pixels of a row; the
+# work-item streams come from oracle.pt_trace (the oracle's BVH traversal over
+# the scene image sr_scene_build writes), sampled over PT_SAMPLE warps spread
+# over the frame
+PT_SAMPLE = 48
+_pt_cache = {}
+
+
+def _pt_streams():
+    if "ops" not in _pt_cache:
+        from paper_conf_cgo_damanijskymg20_b200 import sr
+        c = I.C4
+        tris, mat, mats, cam = I.cornell_scene(c)
+        img = sr.scene_image_host(tris, mat, mats, cam)
+        n_warps = c.n_pixels // 32
+        picks = np.linspace(0, n_warps - 1, PT_SAMPLE).astype(np.int64)
+        pix = (picks[:, None] * 32 + np.arange(32)[None, :]).ravel().astype(np.uint32)
+        ops, off, _ = oracle.pt_trace(img, c.width, c.height, c.spp, c.max_depth,
+                                      I.PRIMARY_SEED, pixels=pix)
+        _pt_cache.update(ops=ops, off=off)
+    return _pt_cache["ops"], _pt_cache["off"]
+
+
+def pt_warps(mode, T=0, U=8):
+    ops, off = _pt_streams()
+    for w in range(PT_SAMPLE):
+        o = off[32 * w:32 * w + 33]
+        yield oracle.ws_pt(ops[o[0]:o[-1]], o - o[0], mode, T, U), 32
+
+
 # the bench launch of configs[2] (dynamic claiming): a persistent grid of
 # 2 x 148 CTAs of 640 threads = 5920 warps, each taking ~10^7 / 5920 photons in
 # chunks from one counter.  Which photons a warp gets depends on timing; their
@@ -191,6 +221,9 @@ CASES = {
     "divloop_pool(T=16)": (r"divloop_poolILi125ELb0", lambda: divloop_pool_warps(1)),
     "divloop_pool_split4(T=16)": (r"divloop_pool_splitILi125ELb0ELi4",
                                   lambda: divloop_pool_warps(4)),
+    "pt_pdom": (r"pt_pdomILb0E", lambda: pt_warps(oracle.PDOM)),
+    f"pt_spec(T={I.C4.threshold})": (r"pt_specILb0ELb1ELb1ELb0E",
+                                      lambda: pt_warps(oracle.SPEC_LOOP, I.C4.threshold, 8)),
     "mcml_pdom": (r"mcml_pdomILb1ELb0ELb1", lambda: mcml_dyn_warps(oracle.PDOM, 0)),
     "mcml_spec(T=32)": (r"mcml_specILb1ELb0ELb1", lambda: mcml_dyn_warps(oracle.SPEC_LOOP, 32)),
 }
@@ -200,11 +233,13 @@ def inst_scale(label):
     """the sampled-warp cases predict instructions for sample_warps of the launch"""
     if label in ("mcml_pdom", "mcml_spec(T=32)"):
         return MC_DYN["warps"] / MC_DYN["sample_warps"]
+    if label.startswith("pt_"):
+        return I.C4.n_pixels / 32 / PT_SAMPLE
     return 1.0
 
 
 def main():
-    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_|rs_")
+    costs = sass_regions.kernel_costs("divloop_|commoncall_|mcml_|rs_|pt_")
     measured = json.load(open(os.path.join(ROOT, "profiles", "simt_efficiency.json")))
     rows = {}
     cases = [(k, v[0], v[1]) for k, v in CASES.items()]
