@@ -197,7 +197,11 @@ SR_API int sr_init(int device, void* cuda_stream, void* workspace_dev, size_t wo
  *                    (sum of popc(R); with DIVLOOP advance_unroll > 1 a lane
  *                    may run several prologs in one such round), 0, 0, 0};
  *                   one record per launched warp (warps past n_threads are
- *                   not written)
+ *                   not written).  DIVLOOP with SR_F_POOL: one record per group
+ *                   of 32 threads, {rounds, releases, Expensive() calls run,
+ *                   windows x slices (the batched advances), that x valid
+ *                   lanes, 0, 0, 0}.  PATHTRACE split merge: words 5, 6 =
+ *                   leaf-test releases and their lanes (words 1, 2: node visits)
  *   SR_T_SCRATCH    internal (claim counters)
  * GRID and COUNTERS are contiguous so a multi-GPU caller can reduce them
  * in place as int64 (two's-complement addition = uint64 addition mod 2^64). */

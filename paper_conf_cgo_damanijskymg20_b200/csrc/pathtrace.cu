@@ -517,13 +517,15 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
       const bool leaf = __popc(L) > __popc(I);
       const uint32_t G = leaf ? L : I;
       if (G != 0u && ((uint32_t)__popc(G) >= a.T || R == 0u)) {
+        if constexpr (SCHED) {  // warp-uniform release counters (every lane keeps them)
+          if (leaf) { ++lrel; lrel_lanes += __popc(G); }
+          else { ++rel; rel_lanes += __popc(G); }
+        }
         if ((G >> lane_id()) & 1u) {
           __syncwarp(G);  // @sr-region REL
           if (leaf) {
-            if constexpr (SCHED) { ++lrel; lrel_lanes += __popc(G); }  // @sr-region LREL
             for (uint32_t k = 0; k < a.unroll && tr.na > 0u; ++k) trav_leaf(a, tr, p.o, p.d, st);  // @sr-region LEAF
           } else {
-            if constexpr (SCHED) { ++rel; rel_lanes += __popc(G); }  // @sr-region NREL
             for (uint32_t k = 0; k < a.unroll && tr.na == 0u && tr.node >= 0; ++k)  // @sr-region STEP
               trav_node(a, tr, p.o, st);
           }

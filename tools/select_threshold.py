@@ -16,7 +16,7 @@ simulated in full at their configs[] size.
 
 TEST/EVALUATION INFRASTRUCTURE: uses oracle/ (event streams + simulator).
 
-usage: python tools/select_threshold.py [--what divloop,rsbench,rsfetch,mcml]
+usage: python tools/select_threshold.py [--what divloop,rsbench,rsfetch,mcml,pathtrace]
            [--thresholds 1,2,4,8,16,24,32] [--mc-warps 512] [--mc-iters 64]
            [--unroll 4] [--measured sweep.json ...] [--write out.json]
 """
@@ -67,20 +67,24 @@ def main():
     ap.add_argument("--write", default="")
     a = ap.parse_args()
     Ts = [int(x) for x in a.thresholds.split(",")]
-    costs = sass_regions.kernel_costs("divloop_|mcml_|rs_")
+    costs = sass_regions.kernel_costs("divloop_|mcml_|rs_|pt_")
 
     fams = {}
     if "divloop" in a.what:
         fams["divloop"] = (r"divloop_pdomILi125ELb0", r"divloop_specILi125ELb0",
                            lambda mode, T: sp.divloop_warps(mode, T), I.C1.n_threads * I.C1.iters)
     if "rsbench" in a.what:
-        fams["rsbench"] = (r"rs_pdomILi8ELi0ELb0", r"rs_specILi8ELi0ELb0",
-                           lambda mode, T: sp.rsbench_warps(mode, T),
+        fams["rsbench"] = (r"rs_pdomILi8ELi0ELb0", r"rs_specILi8ELi0ELb0ELb1E",   # warp pool
+                           lambda mode, T: sp.rsbench_warps(mode, T, pool=True),
                            I.NEXT1.n_threads * I.NEXT1.iters)
     if "rsfetch" in a.what:   # the expensive-prolog variant (trip counts are the same)
-        fams["rsfetch"] = (r"rs_pdomILi8ELi256ELb0", r"rs_specILi8ELi256ELb0",
-                           lambda mode, T: sp.rsbench_warps(mode, T),
+        fams["rsfetch"] = (r"rs_pdomILi8ELi256ELb0", r"rs_specILi8ELi256ELb0ELb1E",
+                           lambda mode, T: sp.rsbench_warps(mode, T, pool=True),
                            I.NEXT1.n_threads * I.NEXT1.iters)
+    if "pathtrace" in a.what:   # sampled warps (simt_predict.PT_SAMPLE), split merge U = 8
+        fams["pathtrace"] = (r"pt_pdomILb0E", r"pt_specILb0ELb1ELb1ELb0E",
+                             lambda mode, T: sp.pt_warps(mode, T, 8),
+                             sp.PT_SAMPLE * 32 * I.C4.spp)
     if "mcml" in a.what:
         sample = mc_sample(a.mc_warps, a.mc_iters)
         # the PDOM kernel ignores the unroll; SPEC runs U steps per release
