@@ -340,23 +340,22 @@ def test_divloop_pool_edge_cases(ctx, kw, split):
 @pytest.mark.parametrize("n,iters", [(2000, 64), (77, 130)])
 @pytest.mark.parametrize("split", [1, 2, 4])
 def test_divloop_pool_schedule_closed_form(ctx, n, iters, split):
-    """per window and slice (64 / split iterations): one batched advance of every
-    valid lane, then ceil(N/32) releases running the slice's N wanted calls"""
+    """per window: one batched advance per slice (64 / split iterations) of every
+    valid lane, then ceil(N/32) releases running the window's N wanted calls
+    (split = 1: the warp's queue; split > 1: the CTA's, dealt to its warps)"""
     w = sr.divloop_workload(flags=sr.F_SCHED | sr.F_POOL, block=64, batch=64, split=split)
     run_divloop(ctx, w, n, iters, I.PRIMARY_SEED, sr.SPEC_LOOP, 16)
     sched = ctx.region(w, n, sr.T_SCHED, torch.int32).view(-1, sr.SCHED_WORDS).cpu().numpy()
     want = oracle.divloop_wants(0, n, iters, I.PRIMARY_SEED)
-    L = 64 // split
     for wi in range((n + 31) // 32):
         ww = want[32 * wi:32 * wi + 32]
         nv = len(ww)
-        Ns = [int(ww[:, b + s * L:min(b + (s + 1) * L, b + 64, iters)].sum())
-              for b in range(0, iters, 64) for s in range(split)]
+        Ns = [int(ww[:, b:min(b + 64, iters)].sum()) for b in range(0, iters, 64)]
         rel = sum((N + 31) // 32 for N in Ns)
         g = sched[wi]
         assert g[1] == rel and g[2] == sum(Ns), wi
-        assert g[3] == len(Ns) and g[4] == len(Ns) * nv, wi
-        assert g[0] == rel + len(Ns), wi
+        assert g[3] == len(Ns) * split and g[4] == len(Ns) * split * nv, wi
+        assert g[0] == rel + len(Ns) * split, wi
 
 
 # ------------------------------------------------------------------ config 2

@@ -40,6 +40,10 @@ timeout 300 $SC -k regex:mcml -o $O/src_mc_pdom_$TAG $OL $MCS --modes pdom --unr
 timeout 300 $SC -k regex:mcml -o $O/src_mc_spec32_$TAG $OL $MCS --modes spec --threshold 32 --unroll 1 > /dev/null 2>&1
 timeout 300 $SC -k regex:mcml -o $O/src_mc_spec8_$TAG $OL $MCS --modes spec --threshold 8 --unroll 1 > /dev/null 2>&1
 timeout 300 $SC -k regex:mcml -o $O/src_mc_spec32u4_$TAG $OL $MCS --modes spec --threshold 32 --unroll 4 > /dev/null 2>&1
+timeout 300 $SC -k regex:divloop_pool -o $O/src_dlpool_$TAG $OL divloop --dl-batch 64 --dl-flags 32 --modes spec > /dev/null 2>&1
+timeout 300 $SC -k regex:divloop_pool -o $O/src_dlpool4_$TAG $OL divloop --dl-batch 64 --dl-flags 32 --dl-split 4 --modes spec > /dev/null 2>&1
+timeout 600 $SC -k regex:pt_pdom -o $O/src_pt_pdom_$TAG $OL pathtrace --modes pdom > /dev/null 2>&1
+timeout 600 $SC -k regex:pt_spec -o $O/src_pt_spec_$TAG $OL pathtrace --modes spec > /dev/null 2>&1
 # full captures of the path tracer kernels (PDOM and the default split merge)
 # (one kernel per process: a second full capture in the same process came back mostly NaN)
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:pt_pdom -c 1 -o $O/prof_ptpdom_$TAG $OL pathtrace --modes pdom > $O/prof_pt_$TAG.log 2>&1

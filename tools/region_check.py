@@ -38,6 +38,8 @@ REPORTS = {
     "rs_pdom": "rs_pdom", "rs_spec(T=32)": "rs_spec",
     "mcml_pdom_static": "mc_pdom", "mcml_spec_static(T=32)": "mc_spec32",
     "mcml_spec_static(T=8)": "mc_spec8", "mcml_spec_static(T=32,U=4)": "mc_spec32u4",
+    "divloop_pool(T=16)": "dlpool", "divloop_pool_split4(T=16)": "dlpool4",
+    "pt_pdom": "pt_pdom", "pt_spec(T=12)": "pt_spec",
 }
 
 
@@ -98,12 +100,13 @@ def predicted_regions(label, costs_all):
             a = acc.setdefault(key, [0.0, 0.0])
             a[0] += c * x
             a[1] += c * l
-    return acc
+    sc = sp.inst_scale(label)   # sampled-warp cases: scale to the whole launch
+    return {k: [v[0] * sc, v[1] * sc] for k, v in acc.items()}
 
 
 def main():
     tag = sys.argv[1]
-    costs_all = sass_regions.kernel_costs("divloop_|mcml_|rs_")
+    costs_all = sass_regions.kernel_costs("divloop_|mcml_|rs_|pt_")
     out = {}
     for label in REPORTS:
         rep = os.path.join(ROOT, "gpurun_out", f"src_{REPORTS[label]}_{tag}.ncu-rep")

@@ -77,10 +77,12 @@ def divloop_warps(mode, T, V=None, batch=False):
 
 
 def divloop_pool_warps(split=1):
-    """the SR_F_POOL kernels: per window and slice (64 / split iterations) of a
-    group of 32 threads, one warp runs the slice's prologs (MASKGRP, 8 draws per
-    group) and ceil(N/32) releases of its N wanted calls (STEP: N lanes in all);
-    warp 0 then adds every thread's results in order (EPIK: as many trips as the
+    """the SR_F_POOL kernels: per window, every (valid) lane runs its prologs
+    (MASKGRP: groups of 8 draws; with split > 1 each of the group's `split` warps
+    takes 64 / split iterations); the window's N wanted calls then run as
+    ceil(N/32) releases (STEP: N lanes in all) -- one warp's queue (split = 1) or
+    the CTA's, its 32-call chunks dealt round-robin to the warps; warp 0 adds
+    every thread's results in order (EPIK: per slice as many trips as the
     thread with the most calls, one lane per call).  Closed-form counts."""
     c = I.C1
     want = oracle.divloop_wants(0, c.n_threads, c.iters, I.PRIMARY_SEED, c.p_u32)
@@ -88,24 +90,28 @@ def divloop_pool_warps(split=1):
     for w in range(0, c.n_threads, 32):
         ww = want[w:w + 32].astype(np.int64)
         nv = len(ww)
-        for sl in range(split):
-            rel = lanes = groups = 0
-            epik_x = epik_l = 0
-            for b in range(0, c.iters, 64):
+        rel = [0] * split
+        lanes = [0] * split
+        groups = [0] * split
+        epik_x = epik_l = 0
+        for b in range(0, c.iters, 64):
+            Ns = []
+            for sl in range(split):
                 lo, hi = b + sl * L, min(b + (sl + 1) * L, b + 64, c.iters)
                 cnt = ww[:, lo:hi].sum(1) if hi > lo else np.zeros(nv, np.int64)
-                N = int(cnt.sum())
-                rel += (N + 31) // 32
-                lanes += N
-                groups += (max(hi - lo, 0) + 7) // 8
-                if sl == 0:   # warp 0 adds every slice's results
-                    for s2 in range(split):
-                        l2, h2 = b + s2 * L, min(b + (s2 + 1) * L, b + 64, c.iters)
-                        c2 = ww[:, l2:h2].sum(1) if h2 > l2 else np.zeros(nv, np.int64)
-                        epik_x += int(c2.max()) if nv else 0
-                        epik_l += int(c2.sum())
-            yield {"MASKGRP": (groups, groups * nv), "RELEASE": (rel, 32 * rel),
-                   "STEP": (rel, lanes), "EPIK": (epik_x, epik_l), "rounds": rel}, nv
+                Ns.append(int(cnt.sum()))
+                groups[sl] += (max(hi - lo, 0) + 7) // 8
+                epik_x += int(cnt.max()) if nv else 0
+                epik_l += int(cnt.sum())
+            N = sum(Ns)
+            chunks = (N + 31) // 32
+            for ch in range(chunks):       # chunk ch -> warp ch % split
+                rel[ch % split] += 1
+                lanes[ch % split] += min(32, N - 32 * ch)
+        for sl in range(split):
+            yield {"MASKGRP": (groups[sl], groups[sl] * nv), "RELEASE": (rel[sl], 32 * rel[sl]),
+                   "STEP": (rel[sl], lanes[sl]),
+                   "EPIK": (epik_x, epik_l) if sl == 0 else (0, 0), "rounds": rel[sl]}, nv
 
 
 def commoncall_warps(mode):
