@@ -52,7 +52,7 @@ NEXT1 = RSBench()
 # Fig. 9's XSBench case: an expensive task fetch (2048 FMAs per
 # lookup prolog, ~0.6x the mean inner-loop work of a lookup) -- refilling idle
 # lanes often no longer pays, the best threshold drops
-NEXT1_FETCH = RSBench(prolog_fma=2048, threshold=16)   # best of the pool sweep (static: 12)
+NEXT1_FETCH = RSBench(prolog_fma=2048, threshold=20)   # best of the pool sweep r02h (static: 12)
 
 
 # (n, mua [1/cm], mus [1/cm], g, d [cm]) -- a synthetic 3-layer tissue slab
