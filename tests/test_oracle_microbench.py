@@ -103,3 +103,51 @@ def test_commoncall_iters_accumulate():
     y1, _ = oracle.commoncall(0, 50, 1, 9)
     y2, _ = oracle.commoncall(0, 50, 2, 9)
     assert np.all(y2 > y1)
+
+
+def test_divloop_per_thread_sums_match_float64_closed_form():
+    """Every thread's (acc, cnt) re-derived in float64 from the definition
+    (reading R3: condition u0 < p_u32 of the thread's Philox draw at event i,
+    Expensive() of U01(u1) by the recurrence's closed form, acc the in-order sum):
+    cnt exactly, acc within the accumulated binary32 rounding bound."""
+    c = I.C1
+    t0, n, seed = 12345, 256, I.PRIMARY_SEED
+    acc, cnt = oracle.divloop(t0, n, c.iters, seed, c.p_u32, c.fma_count)
+    key = [seed & 0xFFFFFFFF, seed >> 32]
+    for j in range(n):
+        t = t0 + j
+        a64, k, mag = 0.0, 0, 0.0
+        for i in range(c.iters):
+            u = oracle.philox([i, 1 << 16, t & 0xFFFFFFFF, t >> 32], key)
+            if int(u[0]) < c.p_u32:
+                r = expensive_closed_form((int(u[1]) >> 8) * 2.0**-24, c.fma_count)
+                a64 += r
+                mag += abs(a64)
+                k += 1
+        assert cnt[j] == k, j
+        # each call within expensive_tol, each of the k additions within 2^-24 |acc|
+        bound = k * expensive_tol(c.fma_count) + mag * 2.0**-24
+        assert abs(float(acc[j]) - a64) <= bound, (j, float(acc[j]), a64, bound)
+
+
+def test_commoncall_per_thread_matches_float64_definition():
+    """Every thread's y re-derived in float64 from reading R4: then-arm iff
+    u0 < split_u32, y = foo(x) with x = U01(u1); else y = foo(fl(fl(x/2) + 1/4))^2
+    (the argument's two binary32 roundings are exact here), foo by the closed form."""
+    c = I.C2
+    t0, n, seed = 99, 300, I.PRIMARY_SEED
+    y, arm = oracle.commoncall(t0, n, 1, seed, c.split_u32, c.fma_count)
+    key = [seed & 0xFFFFFFFF, seed >> 32]
+    tol = expensive_tol(c.fma_count)
+    for j in range(n):
+        t = t0 + j
+        u = oracle.philox([0, 2 << 16, t & 0xFFFFFFFF, t >> 32], key)
+        x = (int(u[1]) >> 8) * 2.0**-24
+        then = int(u[0]) < c.split_u32
+        assert bool(arm[j]) == then, j
+        if then:
+            want, bound = expensive_closed_form(x, c.fma_count), tol
+        else:
+            r = expensive_closed_form(x * 0.5 + 0.25, c.fma_count)
+            want, bound = r * r, 2 * abs(r) * tol + r * r * 2.0**-23
+        assert abs(float(y[j]) - want) <= bound, (j, float(y[j]), want, bound)

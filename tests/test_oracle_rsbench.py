@@ -77,3 +77,40 @@ def test_expensive_prolog_changes_energies_not_trips():
     assert per.min() >= lo * (1 - 1e-5) and per.max() <= hi * (1 + 1e-5)
     acc_plain, _ = oracle.rsbench(0, n, it, 3, fma_count=64)
     assert not np.array_equal(acc, acc_plain)
+
+
+def test_per_thread_sums_match_float64_definition():
+    """Each thread's (acc, nuclides) re-derived from the definition (reading R8):
+    lookup k draws Philox(k, RS<<16, thread); material = the first whose cumulative
+    probability threshold floor(2^32 sum p) exceeds u0 (thresholds recomputed here
+    from the published probabilities); E = U01(u1); nuclide j of material m is
+    (37m + 13j) mod 355 and its body is Expensive() of fl(E + nuc/512) by the
+    recurrence's closed form; acc is the in-order sum.  Nuclides exactly, acc
+    within the accumulated binary32 rounding bound."""
+    thr, cum = [], 0.0
+    for i, p in enumerate(PROB):
+        cum += p
+        thr.append(2**32 - 1 if i == len(PROB) - 1 else math.floor(cum * 2**32))
+    t0, n, iters, seed = 777, 64, 6, I.PRIMARY_SEED
+    acc, nuc = oracle.rsbench(t0, n, iters, seed)
+    key = [seed & 0xFFFFFFFF, seed >> 32]
+    fma = 64
+    for j in range(n):
+        t = t0 + j
+        a64, nn, mag = 0.0, 0, 0.0
+        for k in range(iters):
+            u = oracle.philox([k, 5 << 16, t & 0xFFFFFFFF, t >> 32], key)
+            m = next(i for i, th in enumerate(thr) if int(u[0]) < th) if int(u[0]) < thr[-1] \
+                else len(thr) - 1
+            E = np.float32((int(u[1]) >> 8) * 2.0**-24)
+            xs = 0.0
+            for i in range(NUCS[m]):
+                nid = (37 * m + 13 * i) % 355
+                start = float(np.float32(E + np.float32(nid * 2.0**-9)))
+                xs += expensive_closed_form(start, fma)
+            a64 += xs
+            mag += abs(xs) * NUCS[m] + abs(a64)
+            nn += NUCS[m]
+        assert nuc[j] == nn, j
+        bound = nn * expensive_tol(fma) + mag * 2.0**-24
+        assert abs(float(acc[j]) - a64) <= bound, (j, float(acc[j]), a64, bound)
