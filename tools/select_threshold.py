@@ -82,7 +82,7 @@ def main():
                            lambda mode, T: sp.rsbench_warps(mode, T, pool=True),
                            I.NEXT1.n_threads * I.NEXT1.iters)
     if "pathtrace" in a.what:   # sampled warps (simt_predict.PT_SAMPLE), split merge U = 8
-        fams["pathtrace"] = (r"pt_pdomILb0E", r"pt_specILb0ELb1ELb1ELb0E",
+        fams["pathtrace"] = (r"pt_pdomILb0E", r"pt_specILb0ELb1ELb1ELb0EE",
                              lambda mode, T: sp.pt_warps(mode, T, 8),
                              sp.PT_SAMPLE * 32 * I.C4.spp)
     if "mcml" in a.what:
