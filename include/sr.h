@@ -276,12 +276,17 @@ SR_API int sr_math_eval(int fn, const float* x_dev, float* out_dev, uint64_t n);
  *   SR_FNP_HG_SINT   sqrt(1 - cos(theta)^2) of the same
  *   SR_FNP_DIV2_XP   (x[2j], x[2j+1]) / p as one f32x2 pair (div2_dom, the
  *                    rotation's two quotients)
+ *   SR_FNP_FRESNEL + v, v in [0, 8): MCML's Fresnel sub-step for cos(incidence)
+ *                    = x at indices (ni, nt) = (p, 1) (v bit 2 clear) or (1, p)
+ *                    (set); the reflectance (v bit 1 clear) or the transmitted
+ *                    cosine ca2 (set); the FAST kernels' operations (v bit 0 set)
+ *                    or the guarded IEEE ones (clear)
  * Each equals the IEEE binary32 result bit for bit on the domain its call
  * site guarantees; outside it the result is unspecified.
  * Errors: SR_E_STATE before sr_init; SR_E_INVALID (unknown fn, NULL with
  * n > 0); SR_E_CUDA. */
 enum { SR_FNP_DIV_XP = 0, SR_FNP_DIV_PX = 1, SR_FNP_SQRT = 2, SR_FNP_HG_COST = 3,
-       SR_FNP_HG_SINT = 4, SR_FNP_DIV2_XP = 5 };
+       SR_FNP_HG_SINT = 4, SR_FNP_DIV2_XP = 5, SR_FNP_FRESNEL = 8 };
 SR_API int sr_math_eval_p(int fn, float p, const float* x_dev, float* out_dev, uint64_t n);
 
 /* Diagnostics: closest hit of n rays against a scene built by sr_scene_build,

@@ -196,11 +196,15 @@ int sr_math_eval(int fn, const float* x_dev, float* out_dev, uint64_t n) {
 int sr_math_eval_p(int fn, float p, const float* x_dev, float* out_dev, uint64_t n) {
   std::lock_guard<std::mutex> lk(g_mu);
   g_err.clear();
-  if (fn < SR_FNP_DIV_XP || fn > SR_FNP_DIV2_XP) return fail(SR_E_INVALID, "unknown fn");
+  const bool fres = fn >= SR_FNP_FRESNEL && fn < SR_FNP_FRESNEL + 8;
+  if (!fres && (fn < SR_FNP_DIV_XP || fn > SR_FNP_DIV2_XP)) return fail(SR_E_INVALID, "unknown fn");
   if (n && (!x_dev || !out_dev)) return fail(SR_E_INVALID, "NULL array");
   if (!g_ctx.live) return fail(SR_E_STATE, "sr_math_eval_p before sr_init");
   if (!n) return SR_OK;
-  const cudaError_t e = launch_math_eval_p(g_ctx.stream, g_ctx.sm_count, fn, p, x_dev, out_dev, n);
+  const cudaError_t e =
+      fres ? launch_fresnel_eval(g_ctx.stream, g_ctx.sm_count, fn - SR_FNP_FRESNEL, p, x_dev,
+                                 out_dev, n)
+           : launch_math_eval_p(g_ctx.stream, g_ctx.sm_count, fn, p, x_dev, out_dev, n);
   if (e != cudaSuccess) return fail_cuda(e, "sr_math_eval_p");
   return SR_OK;
 }

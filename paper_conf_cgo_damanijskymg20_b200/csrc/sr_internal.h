@@ -64,6 +64,8 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
 
 cudaError_t launch_math_eval(cudaStream_t st, int sm_count, int fn, const float* x, float* out,
                              uint64_t n);
+cudaError_t launch_fresnel_eval(cudaStream_t st, int sm_count, int variant, float p,
+                                const float* x, float* out, uint64_t n);
 cudaError_t launch_math_eval_p(cudaStream_t st, int sm_count, int fn, float p, const float* x,
                                float* out, uint64_t n);
 cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* rays, int64_t* hit,

@@ -30,7 +30,7 @@ EXPORTS = ["sr_init", "sr_workspace_bytes", "sr_workspace_region", "sr_run", "sr
            "sr_math_eval_p", "sr_pt_closest", "sr_scene_build", "sr_scene_build_host"]
 PT_COUNTERS = ["paths", "rays", "node_visits", "tri_tests"]
 FN_LOGF, FN_SIN2PI, FN_COS2PI, FN_EXPENSIVE_1000, FN_EXPENSIVE_2000 = 0, 1, 2, 3, 4
-FNP_DIV_XP, FNP_DIV_PX, FNP_SQRT, FNP_HG_COST, FNP_HG_SINT, FNP_DIV2_XP = 0, 1, 2, 3, 4, 5
+FNP_DIV_XP, FNP_DIV_PX, FNP_SQRT, FNP_HG_COST, FNP_HG_SINT, FNP_DIV2_XP, FNP_FRESNEL = 0, 1, 2, 3, 4, 5, 8
 
 
 class SRError(RuntimeError):

@@ -96,6 +96,33 @@ def test_div_dom_path_length_every_rng_input(ctx, mut):
     assert_bits(got, (-lg) / F32(mut), lg)
 
 
+@pytest.mark.parametrize("n", [1.4, 1.33, 1.5, 1.0 + 2.0**-10, 2.0**10, 2.0**-10, 1.0 - 2.0**-10])
+def test_fresnel_fast_path_every_cosine(ctx, n):
+    """MCML's Fresnel sub-step on the FAST kernels' div_dom / sqrt_dom == the IEEE
+    operations, reflectance and transmitted cosine, for EVERY binary32 cos(incidence)
+    in [0, 1], both directions (into and out of the denser medium), at the indices
+    of configs[2] (1.4 | 1) and at the edges of mc_fast_domain (ratio 1 + 2^-10,
+    n = 2^10 and 2^-10)."""
+    total = 0x3F800000 + 1                       # bit patterns of +0 .. 1.0
+    chunk = 1 << 26
+    for rev in (0, 4):
+        for what in (0, 2):                      # reflectance, ca2
+            for b in range(0, total, chunk):
+                bits = torch.arange(b, min(b + chunk, total), dtype=torch.int64, device="cuda")
+                x = bits.to(torch.int32).view(torch.float32)
+                fast, ieee = torch.empty_like(x), torch.empty_like(x)
+                p = float(np.float32(n))
+                sr.sr_math_eval_p(sr.FNP_FRESNEL + 1 + what + rev, p, x.data_ptr(), fast.data_ptr(),
+                                  x.numel())
+                sr.sr_math_eval_p(sr.FNP_FRESNEL + what + rev, p, x.data_ptr(), ieee.data_ptr(),
+                                  x.numel())
+                ctx.stream.synchronize()
+                bad = (fast.view(torch.int32) != ieee.view(torch.int32)).nonzero()
+                assert bad.numel() == 0, (n, rev, what, int(bad.numel()),
+                                          x[bad[:5, 0]].tolist(), fast[bad[:5, 0]].tolist(),
+                                          ieee[bad[:5, 0]].tolist())
+
+
 @pytest.mark.parametrize("p", [3.0, -0.37, 2.0**-40, 2.0**40, 1.0 + 2.0**-23])
 def test_div_dom_log_uniform_operands(ctx, p):
     """x / p and p / x for 2^22 operands of both signs, log-uniform over [2^-60, 2^60]."""
