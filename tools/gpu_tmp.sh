@@ -1,5 +1,12 @@
 python -c "import __graft_entry__ as g; g.build()"
 O=gpurun_out
-timeout 900 python -m pytest tests/test_gpu_parity.py -q -k "fresnel" > $O/t_g18.log 2>&1; tail -15 $O/t_g18.log
-timeout 1800 python -m pytest tests/test_gpu_parity.py tests/test_gpu_fullsize.py -q -x -k "mcml or fullsize or full_config or outside" > $O/t_g18b.log 2>&1; tail -2 $O/t_g18b.log
-for i in 1 2; do timeout 300 python bench.py --no-cpu --no-configs --steps 10 > $O/b18_$i.json 2>/dev/null; python tools/bench_summary.py $O/b18_$i.json; done
+python tools/build_variants.py libsr_ptl4.so libsr_ptl16.so libsr_ptl2.so > /dev/null 2>&1
+for L in libsr.so libsr_ptl2.so libsr_ptl4.so libsr_ptl16.so; do
+  SR_LIB=paper_conf_cgo_damanijskymg20_b200/$L timeout 900 python tools/sweep.py --what pathtrace --thresholds 10,12,14 --unroll 8 --reps 3 > $O/sw_ptl_$L.json 2>/dev/null
+  python -c "
+import json;d=json.load(open('$O/sw_ptl_$L.json'))['pathtrace']
+print('$L', [(r['mode'],r['T'],round(r['ms'],2)) for r in d])"
+done
+for U in 6 10 12; do timeout 900 python tools/sweep.py --what pathtrace --thresholds 10,12,14 --unroll $U --reps 3 > $O/sw_ptu_$U.json 2>/dev/null; python -c "
+import json;d=json.load(open('$O/sw_ptu_$U.json'))['pathtrace']
+print('U=$U', [(r['mode'],r['T'],round(r['ms'],2)) for r in d])"; done
