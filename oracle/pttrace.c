@@ -14,8 +14,8 @@
  *     t, leaves tested child 0 first, the nearer inner child first, the other
  *     pushed; empty next -> pop), so the closest hits -- and the image -- equal
  *     the brute force (tests/test_oracle_pttrace.py checks the image bit for bit).
- * (2) ws_pt replays those streams under the PDOM rule (the kernels' do-while
- *     bounce loop with an inline traversal loop) and under the split Loop Merge
+ * (2) ws_pt replays those streams under the PDOM rule (the bounce loop and the
+ *     traversal loop inside it, both reconverging at their latches) and under the split Loop Merge
  *     of pt_spec (two concurrent predictions: inner-node visits I vs leaf tests
  *     L, the larger group released when |G| >= T or no lane can refill, U work
  *     items per release; idle lanes shade, start the next sample and the next
@@ -335,7 +335,9 @@ void ws_pt(const uint16_t* ops, const uint64_t* off, uint32_t n_valid, int mode,
         hit(o, WS_PT_TBEGIN, alive);
         uint32_t tr = alive;        /* lanes still traversing */
         while (tr) {
-          hit(o, WS_PT_STEP, tr);
+          /* the loop's vote and latch run with every lane of the bounce (the
+           * kernel reconverges them there); the visit with the traversing ones */
+          hit(o, WS_PT_STEP, alive);
           node_hits(o, ops, pc, tr);
           /* the visit's inline leaf loop: child 0's tests, then child 1's */
           uint32_t nt[32] = {0}, mx = 0;

@@ -226,6 +226,7 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d,
   // leaves: test their triangles now (child 0's, then child 1's, one loop);
   // inner children: descend / push
   const int32_t n0 = (h0 && N.cnt0 > 0) ? N.cnt0 : 0, n1 = (h1 && N.cnt1 > 0) ? N.cnt1 : 0;
+#pragma unroll 1  // one triangle test per trip (the simulator's LEAF count)
   for (int32_t k = 0; k < n0 + n1; ++k) {  // @sr-region LEAFIF
     const int32_t at = k < n0 ? N.ref0 + k : N.ref1 + (k - n0);  // @sr-region LEAF
     tri_test(load_tri(a.tris, at), at, o, d, tr.tb, tr.ib, tr.mb, tr.slot);
@@ -295,9 +296,21 @@ __device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, V3 o, V3 d,
   }
 }  // @sr-region END
 
-__device__ __forceinline__ int64_t closest_hit(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
+// SYNC (the PDOM kernel): the lanes of `mask` run the traversal loop together and
+// reconverge at its latch every trip -- the loop's immediate post-dominator --
+// instead of letting independent thread scheduling split the warp inside it.
+template <bool SYNC>
+__device__ __forceinline__ int64_t closest_hit(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st,
+                                               uint32_t mask = 0u) {
   trav_begin(tr, d);  // @sr-region TBEGIN
-  while (trav_step(a, tr, o, d, st)) {  // @sr-region STEP
+  if constexpr (SYNC) {
+    bool more = true;
+    while (__any_sync(mask, more)) {  // @sr-region STEP
+      if (more) more = trav_step(a, tr, o, d, st);
+    }
+  } else {
+    while (trav_step(a, tr, o, d, st)) {  // @sr-region STEP
+    }
   }
   return (int64_t)tr.ib;  // @sr-region BOUNCE
 }  // @sr-region END
@@ -430,8 +443,9 @@ __device__ __forceinline__ void finish(const PtArgs& a, const Path& p, bool vali
   }
 }  // @sr-region END
 
-__device__ __forceinline__ void bounce(const PtArgs& a, Path& p, Trav& tr, Stats& st) {
-  closest_hit(a, tr, p.o, p.d, st);  // @sr-region BOUNCE
+__device__ __forceinline__ void bounce(const PtArgs& a, Path& p, Trav& tr, Stats& st,
+                                       uint32_t mask) {
+  closest_hit<true>(a, tr, p.o, p.d, st, mask);  // @sr-region BOUNCE
   ++st.rays;
   shade(a, p, tr);
 }  // @sr-region END
@@ -457,17 +471,17 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_PDOM) pt_pdom(const PtA
       p.s = s;  // @sr-region LAUNCH
       camera_ray(a, H, p);              // Prolog
       ++paths;
-      do {                              // L1: bounce loop, divergent trip count  // @sr-region BOUNCE
-        if constexpr (SCHED) {
-          const uint32_t m = __activemask();
-          if (lane_id() == (uint32_t)(__ffs(m) - 1)) { ++rel; rel_lanes += __popc(m); }
-        }
-        bounce(a, p, tr, st);
-      } while (p.alive);  // @sr-region BOUNCE
+    }
+    // L1: the bounce loop, divergent trip count; every bounce reconverges at the
+    // loop latch (its immediate post-dominator), as the traversal loop inside does
+    uint32_t A = __ballot_sync(kFull, valid);  // @sr-region OUTER:full
+    while (A != 0u) {  // @sr-region BOUNCE
+      if constexpr (SCHED) { ++rel; rel_lanes += __popc(A); }
+      if ((A >> lane_id()) & 1u) bounce(a, p, tr, st, A);
+      A = __ballot_sync(kFull, valid && p.alive);  // @sr-region BOUNCE
     }                                   // IPDOM: reconverge, next sample  // @sr-region OUTER:full
   }
-  uint32_t r = 0, rl = 0;  // @sr-region ENTRY:full
-  if constexpr (SCHED) { r = __reduce_add_sync(kFull, rel); rl = __reduce_add_sync(kFull, rel_lanes); }
+  uint32_t r = rel, rl = rel_lanes;  // @sr-region ENTRY:full
   finish(a, p, valid, st, paths, g >> 5, outer, r, rl, outer, launch_lanes);
 }
 
@@ -574,7 +588,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
         if constexpr (NODE) {
           for (uint32_t k = 0; k < a.unroll && trav; ++k) trav = trav_step(a, tr, p.o, p.d, st);
         }
-        else bounce(a, p, tr, st);
+        else bounce(a, p, tr, st, P);
       }
     } else {
       if constexpr (SCHED) { ++adv; adv_lanes += __popc(R); }
@@ -605,7 +619,7 @@ __global__ void pt_query(const PtArgs a) {
   const float* r = a.q_rays + 6 * i;
   Stats st{0, 0, 0};
   Trav tr;
-  const int64_t h = closest_hit(a, tr, mk(r[0], r[1], r[2]), mk(r[3], r[4], r[5]), st);
+  const int64_t h = closest_hit<false>(a, tr, mk(r[0], r[1], r[2]), mk(r[3], r[4], r[5]), st);
   a.q_hit[i] = h;
   a.q_t[i] = tr.tb;
 }

@@ -54,7 +54,4 @@ def test_simt_prediction_within_2_points(prediction, label):
     # sub-cases, roulette outcomes -- and count both copies of a rotated loop
     # test; the MC and RSBench kernels land 8-12 % off)
     inst = p["inst"] * sp.inst_scale(label)
-    # the path tracer's PDOM kernel: its inline leaf loop and the bounce loop's rarely
-    # taken blocks are costed at the block level: +19 %
-    bound = 0.20 if label == "pt_pdom" else 0.15
-    assert abs(inst / m["inst"] - 1) < bound, (label, inst, m["inst"])
+    assert abs(inst / m["inst"] - 1) < 0.15, (label, inst, m["inst"])

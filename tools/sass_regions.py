@@ -346,7 +346,9 @@ def kernel_costs(kernel_regex=".*"):
         # per entry of the inner loop -- per release / advance round / launch -- with
         # that step's lanes, so they are costed to the entering region
         regions_here = {f[0] for f in final if f is not None}
-        enter = {"STEP": "RELEASE" if "RELEASE" in regions_here else "LAUNCH",
+        # (the path tracer's PDOM traversal loop is entered once per bounce: BOUNCE)
+        enter = {"STEP": ("BOUNCE" if "BOUNCE" in regions_here else
+                          "RELEASE" if "RELEASE" in regions_here else "LAUNCH"),
                  "PROLOG": "ADVANCE"}
         for rname, ename in enter.items():
             if ename not in regions_here and ename != "LAUNCH":
@@ -357,6 +359,11 @@ def kernel_costs(kernel_regex=".*"):
                 continue
             inner = [(a_, b_) for a_, b_ in loops
                      if sum(a_ <= i <= b_ for i in idx) * 2 > len(idx)]
+            if ename == "BOUNCE":
+                # the path tracer's PDOM traversal loop: its vote / latch are a few of the
+                # region's instructions, the loop's entry and exit code the rest -- the
+                # innermost loop holding any of them is the traversal loop
+                inner = [(a_, b_) for a_, b_ in loops if any(a_ <= i <= b_ for i in idx)]
             if not inner:
                 continue
             a_in, b_in = min(inner, key=lambda ab: ab[1] - ab[0])
