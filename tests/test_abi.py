@@ -172,7 +172,7 @@ def test_sass_is_sm100a_and_uses_the_intended_instructions():
             assert ops(r"\bVOTE\.", f) >= 2, f          # __ballot_sync scheduler
         if "ILi125ELb0" in f:
             assert ops(r"\bFFMA2\b", f) == 500, f       # 1000 FMAs as FFMA2, unrolled
-        if "mcml_" in f:
+        if re.search(r"\dmcml_(pdom|spec)", f):
             # paired IEEE products only: every FFMA2 adds the -0 pair from the kernel
             # parameters (a uniform register), never a contracted product + sum
             # -- except the three FFMA2 of div2_dom (the rotation's paired quotients,
