@@ -27,6 +27,7 @@ def sources():
 
 def headers():
     return sorted(glob.glob(os.path.join(HERE, "csrc", "*.h*")) +
+                  glob.glob(os.path.join(HERE, "csrc", "*.cuh")) +
                   glob.glob(os.path.join(ROOT, "include", "*.h")))
 
 
