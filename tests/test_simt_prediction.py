@@ -51,7 +51,8 @@ def test_simt_prediction_within_2_points(prediction, label):
     assert abs(p["simt"] - m["simt_efficiency"]) * 100 < 2.0, (label, p["simt"], m["simt_efficiency"])
     # the warp-instruction count itself is predicted too (sanity bound: static
     # costs ignore sub-branches that are rarer than their region -- Fresnel
-    # sub-cases, roulette outcomes -- and count both copies of a rotated loop
-    # test; the MC and RSBench kernels land 8-12 % off)
+    # sub-cases, roulette outcomes, the nuclide loop's window edges -- and count
+    # both arms of a warp-uniform if/else in the region that holds them; every
+    # launch lands within 5 %)
     inst = p["inst"] * sp.inst_scale(label)
-    assert abs(inst / m["inst"] - 1) < 0.15, (label, inst, m["inst"])
+    assert abs(inst / m["inst"] - 1) < 0.06, (label, inst, m["inst"])

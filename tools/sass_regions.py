@@ -351,7 +351,9 @@ def kernel_costs(kernel_regex=".*"):
                           "RELEASE" if "RELEASE" in regions_here else "LAUNCH"),
                  "PROLOG": "ADVANCE"}
         for rname, ename in enter.items():
-            if ename not in regions_here and ename != "LAUNCH":
+            # (ADVANCE has no code of its own when the SCHED counters are compiled
+            # out; the simulator still counts its rounds)
+            if ename not in regions_here and ename not in ("LAUNCH", "ADVANCE"):
                 continue
             idx = [i for i in range(len(body)) if final[i] is not None and final[i][0] == rname
                    and i not in cold]
