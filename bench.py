@@ -635,17 +635,17 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
                      "rays": int(cnt[1]), "node_visits": int(cnt[2]), "tri_tests": int(cnt[3]),
                      "launch": sr.sr_last_launch()}
     res["speedup_vs_pdom"] = res[sname]["value"] / res["pdom"]["value"]
-    # issue roofline (as MC): useful work = the PDOM kernel's thread-instructions per
-    # path (ncu, profiles/simt_efficiency.json), peak = 592 SMSPs x 32 lanes x f
-    simt = load_json(os.path.join(ROOT, "profiles", "simt_efficiency.json")) or {}
-    ti = (simt.get("pt_pdom") or {}).get("thread_inst")
-    if ti:
-        per_path = ti / (c.n_pixels * c.spp)
+    # issue roofline (as MC): useful work = thread-instructions per path of a PDOM
+    # kernel whose lanes each execute only their own path (profiles/work_per_unit.json,
+    # pt_basis), peak = 592 SMSPs x 32 lanes x f
+    per_path = (load_json(PROFILE_CONST) or {}).get("pt_thread_inst_per_path")
+    if per_path:
         peak = 592 * 32 * f_mhz * 1e6
         res["issue_roofline"] = {
             "thread_inst_per_path": per_path,
             "frac": {k: per_path * res[k]["value"] / peak for k in ("pdom", sname)},
-            "basis": "PDOM thread-inst per path (ncu) x paths/s / (592 x 32 x sm_max_mhz)"}
+            "basis": "profiles/work_per_unit.json pt_thread_inst_per_path (ncu, as-compiled "
+                     "PDOM) x paths/s / (592 x 32 x sm_max_mhz)"}
     out["pathtrace"] = res
     return out
 
