@@ -136,6 +136,14 @@ __device__ __forceinline__ PtMat load_mat(const PtMat* base, uint32_t i) {
 
 // Conservative slab test against a padded box: accept when the ray's
 // parametric interval [tmin, tbest] can touch the box (slack 1e-5 relative).
+// Callers evaluate it for both child slots unconditionally and AND the result
+// with `slot is not empty` (no branch around the test: the box arithmetic is
+// cheaper than the divergence bookkeeping of a short-circuit).
+#ifdef SR_PT_BOX_BRANCH  // tuning variant: the short-circuit form
+#define SR_PT_SLOT_TEST(REF, HIT) ((REF) >= 0 && (HIT))
+#else
+#define SR_PT_SLOT_TEST(REF, HIT) ((HIT) & ((REF) >= 0))
+#endif
 __device__ __forceinline__ bool box_hit(const float* lo, const float* hi, V3 o, V3 inv, float tb,
                                         float& tnear) {
   const float tx0 = (lo[0] - o.x) * inv.x, tx1 = (hi[0] - o.x) * inv.x;
@@ -221,8 +229,8 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d,
   const PtNode N = load_node(a.nodes, tr.node);  // @sr-region NODE
   ++st.nodes;
   float tn0, tn1;
-  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0);
-  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1);
+  const bool h0 = SR_PT_SLOT_TEST(N.ref0, box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0));
+  const bool h1 = SR_PT_SLOT_TEST(N.ref1, box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1));
   // leaves: test their triangles now (child 0's, then child 1's, one loop);
   // inner children: descend / push
   const int32_t n0 = (h0 && N.cnt0 > 0) ? N.cnt0 : 0, n1 = (h1 && N.cnt1 > 0) ? N.cnt1 : 0;
@@ -261,8 +269,8 @@ __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats
   const PtNode N = load_node(a.nodes, tr.node);  // @sr-region NODE
   ++st.nodes;
   float tn0, tn1;
-  const bool h0 = N.ref0 >= 0 && box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0);
-  const bool h1 = N.ref1 >= 0 && box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1);
+  const bool h0 = SR_PT_SLOT_TEST(N.ref0, box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0));
+  const bool h1 = SR_PT_SLOT_TEST(N.ref1, box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1));
   const bool l0 = h0 && N.cnt0 > 0, l1 = h1 && N.cnt1 > 0;
   tr.la = l0 ? N.ref0 : N.ref1;
   tr.na = l0 ? (uint32_t)N.cnt0 : (l1 ? (uint32_t)N.cnt1 : 0u);
