@@ -104,10 +104,26 @@ struct Stats {
 // one scalar load per field (the structs are 4-byte aligned, so the compiler
 // would not vectorise them itself; the image keeps every record 16-byte
 // aligned: 128-byte header, 64-byte nodes, 48-byte triangles).
+// sm_100 has 256-bit global loads: a node (64 bytes, 64-byte aligned in the image)
+// is two LDG.E.256 instead of four LDG.E.128 (SR_PT_LDG128 keeps the latter as a
+// tuning variant).
+__device__ __forceinline__ void ldg256(const void* p, float4& a, float4& b) {
+  asm("ld.global.nc.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+      : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
+      : "l"(p));
+}
 __device__ __forceinline__ PtNode load_node(const PtNode* base, int32_t i) {
   const float4* q = reinterpret_cast<const float4*>(base + i);
+#ifdef SR_PT_LDG128
   const float4 x = __ldg(q), y = __ldg(q + 1), z = __ldg(q + 2);
   const int4 w = __ldg(reinterpret_cast<const int4*>(q + 3));
+#else
+  float4 x, y, z, wf;
+  ldg256(q, x, y);
+  ldg256(q + 2, z, wf);
+  const int4 w = make_int4(__float_as_int(wf.x), __float_as_int(wf.y), __float_as_int(wf.z),
+                           __float_as_int(wf.w));
+#endif
   PtNode n;
   n.b0lo[0] = x.x; n.b0lo[1] = x.y; n.b0lo[2] = x.z; n.b0hi[0] = x.w;
   n.b0hi[1] = y.x; n.b0hi[2] = y.y; n.b1lo[0] = y.z; n.b1lo[1] = y.w;

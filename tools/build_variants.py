@@ -29,6 +29,7 @@ VARIANTS = {
     "libsr_pt8.so": ["SR_PT_MINB_SPEC=8", "SR_PT_MINB_PDOM=8"],
     "libsr_pt7.so": ["SR_PT_MINB_SPEC=7", "SR_PT_MINB_PDOM=7"],
     "libsr_ptbb.so": ["SR_PT_BOX_BRANCH"],
+    "libsr_pt128.so": ["SR_PT_LDG128"],
 }
 if __name__ == "__main__":
     names = sys.argv[1:] or list(VARIANTS)
