@@ -69,11 +69,15 @@ __device__ __forceinline__ float energy(const RsArgs& a, uint32_t u1) {
   else return E;
 }
 
+// K: chains_round's addend pairs held in registers by the kernel (chain_addends;
+// compile-time ROUNDS only)
 template <int ROUNDS>
-__device__ __forceinline__ float body(float E, uint32_t m, uint32_t i, uint32_t rounds) {
+__device__ __forceinline__ float body(float E, uint32_t m, uint32_t i, uint32_t rounds,
+                                      const ChainAdd& K) {
   const uint32_t nuc = (37u * m + 13u * i) % kNuclides;
   const float start = E + (float)nuc * 0x1p-9f;
-  return expensive<ROUNDS>(start, rounds);
+  if constexpr (ROUNDS > 0) return expensive_k<ROUNDS>(start, K);
+  else return expensive<0>(start, rounds);
 }
 
 __device__ __forceinline__ void finish(const RsArgs& a, uint64_t g, bool valid, float acc,
@@ -94,6 +98,7 @@ __device__ __forceinline__ void finish(const RsArgs& a, uint64_t g, bool valid, 
 template <int ROUNDS, int PROLOG, bool SCHED>
 __global__ void __launch_bounds__(SR_RS_MAXT) rs_pdom(const RsArgs a) {
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
+  const ChainAdd K = chain_addends(a.rounds - (uint32_t)ROUNDS);  // a.rounds == ROUNDS here
   const bool valid = g < a.n;
   const uint64_t t = a.t0 + g;
   float acc = 0.0f;
@@ -114,7 +119,7 @@ __global__ void __launch_bounds__(SR_RS_MAXT) rs_pdom(const RsArgs a) {
         const uint32_t mk = __activemask();
         if (lane_id() == (uint32_t)(__ffs(mk) - 1)) { ++rel; rel_lanes += __popc(mk); }
       }
-      xs = xs + body<ROUNDS>(E, m, i, a.rounds);
+      xs = xs + body<ROUNDS>(E, m, i, a.rounds, K);
     }
     acc = acc + xs;  // @sr-region LAUNCH:full
     nucs += N;
@@ -128,6 +133,7 @@ template <int ROUNDS, int PROLOG, bool SCHED, bool POOL>
 __global__ void __launch_bounds__(SR_RS_MAXT) rs_spec(const RsArgs a) {
   extern __shared__ float rs_xs[];  // POOL: per warp xs[iters][32], then nucs[32]
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;  // @sr-region ENTRY:full
+  const ChainAdd K = chain_addends(a.rounds - (uint32_t)ROUNDS);  // a.rounds == ROUNDS here
   const bool valid = g < a.n;
   uint64_t t = a.t0 + g;
   float acc = 0.0f, xs = 0.0f, E = 0.0f;
@@ -158,7 +164,7 @@ __global__ void __launch_bounds__(SR_RS_MAXT) rs_spec(const RsArgs a) {
         // up to `unroll` inner iterations per release; a lane whose lookup ends
         // inside the release idles for the rest of it
         for (uint32_t r = 0; r < a.unroll && busy; ++r) {
-          xs = xs + body<ROUNDS>(E, m, i, a.rounds);
+          xs = xs + body<ROUNDS>(E, m, i, a.rounds, K);
           i = i + 1u;
           if (i == N) {                    // inner loop done: Epilog
             if constexpr (POOL) {
