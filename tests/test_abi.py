@@ -104,6 +104,11 @@ def test_run_validation_before_state():
     with pytest.raises(sr.SRError) as e:
         sr.sr_run(sr.divloop_workload(batch=64, block=1024), 64, 1, 1, sr.PDOM, 0)
     assert e.value.code == sr.SR_E_INVALID and "block_threads <= 512" in str(e.value)
+    for split in (3, 5, 8):
+        bad = sr.divloop_workload(batch=64, flags=sr.F_POOL, split=split)
+        with pytest.raises(sr.SRError) as e:
+            sr.sr_run(bad, 64, 64, 1, sr.SPEC_LOOP, 16)
+        assert e.value.code == sr.SR_E_INVALID and "pool_split" in str(e.value)
 
 
 def test_mcml_param_validation():
