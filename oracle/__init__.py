@@ -25,7 +25,7 @@ CFLAGS = ["-O2", "-std=gnu11", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "
           "-Wall", "-Wno-unused-function"]
 
 TAG_DIV, TAG_CALL, TAG_MC, TAG_PT = 1, 2, 3, 4
-PDOM, SPEC_LOOP, SPEC_CALL = 0, 1, 2
+PDOM, SPEC_LOOP, SPEC_CALL, SPEC_LOOP_POOL = 0, 1, 2, 3
 # region ids (oracle.h)
 DL = dict(ENTRY=0, PROLOG=1, EXPENSIVE=2, EPILOG=3, ROUND=4, RELEASE=5, ADVANCE=6)
 CC = dict(ENTRY=0, THEN=1, ELSE_PRE=2, CALL=3, ELSE_POST=4, MERGE=5)
@@ -335,7 +335,8 @@ def pt_trace(img, width, height, spp, max_depth, seed, pixels=None, cap=None):
 
 
 def ws_pt(ops, off, mode, T=0, U=1):
-    """one warp's PDOM / split Loop Merge schedule (off: n_valid + 1 offsets)"""
+    """one warp's PDOM / split Loop Merge schedule (off: n_valid + 1 offsets);
+    mode SPEC_LOOP_POOL: the split merge with the warp's paths pooled"""
     ops = np.ascontiguousarray(ops, np.uint16)
     off = np.ascontiguousarray(off, np.uint64)
     o = WsCounts()

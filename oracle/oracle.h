@@ -159,7 +159,7 @@ void or_rsbench(uint32_t fma_count, uint32_t prolog_fma, uint64_t t0, uint64_t n
                 uint32_t iters, uint64_t seed, float* acc, uint32_t* nuc, uint32_t* trips);
 
 /* ---- warpsim.c : lane-mask warp simulator (oracle part 2). */
-enum { WS_PDOM = 0, WS_SPEC_LOOP = 1, WS_SPEC_CALL = 2 };
+enum { WS_PDOM = 0, WS_SPEC_LOOP = 1, WS_SPEC_CALL = 2, WS_SPEC_LOOP_POOL = 3 };
 /* regions of the divloop program (Listing 1) */
 enum { WS_DL_ENTRY = 0, WS_DL_PROLOG, WS_DL_EXPENSIVE, WS_DL_EPILOG, WS_DL_ROUND,
        WS_DL_RELEASE, WS_DL_ADVANCE, WS_DL_NREG };
@@ -237,7 +237,10 @@ enum { WS_PT_ENTRY = 0, WS_PT_OUTER, WS_PT_LAUNCH, WS_PT_BOUNCE, WS_PT_TBEGIN, W
        WS_PT_SH, WS_PT_SH_HIT, WS_PT_SH_SURF, WS_PT_SH_DIFF, WS_PT_SH_MIRR, WS_PT_SH_GLASS,
        WS_PT_SH_RR, WS_PT_SH_END, WS_PT_ROUND, WS_PT_REL, WS_PT_LREL, WS_PT_NREL, WS_PT_ADV };
 /* the PDOM (mode WS_PDOM) or split Loop Merge (WS_SPEC_LOOP, threshold T, U
- * work items per release) schedule of one warp of n_valid lanes */
+ * work items per release) schedule of one warp of n_valid lanes; WS_SPEC_LOOP_POOL:
+ * the split merge with the warp's n_valid x spp paths claimed from one pool
+ * (spp <= WS_PT_POOL_MAX_SPP) */
+#define WS_PT_POOL_MAX_SPP 64
 void ws_pt(const uint16_t* ops, const uint64_t* off, uint32_t n_valid, int mode, uint32_t T,
            uint32_t U, ws_counts* out);
 

@@ -15,12 +15,13 @@
  *     pushed; empty next -> pop), so the closest hits -- and the image -- equal
  *     the brute force (tests/test_oracle_pttrace.py checks the image bit for bit).
  * (2) ws_pt replays those streams under the PDOM rule (the bounce loop and the
- *     traversal loop inside it, both reconverging at their latches) and under the split Loop Merge
- *     of pt_spec (two concurrent predictions: inner-node visits I vs leaf tests
+ *     traversal loop inside it, both reconverging at their latches) and under the split
+ *     Loop Merge of pt_spec (two concurrent predictions: inner-node visits I vs leaf tests
  *     L, the larger group released when |G| >= T or no lane can refill, U work
  *     items per release; idle lanes shade, start the next sample and the next
- *     ray in advance rounds), counting warp executions and active lanes per
- *     source region (WS_PT_*), as warpsim.c does for the other kernels.
+ *     ray in advance rounds) -- each lane on its own pixel, or (WS_SPEC_LOOP_POOL)
+ *     taking the next path of the warp's pool -- counting warp executions and active
+ *     lanes per source region (WS_PT_*), as warpsim.c does for the other kernels.
  */
 #include <math.h>
 #include <string.h>
@@ -373,11 +374,42 @@ void ws_pt(const uint16_t* ops, const uint64_t* off, uint32_t n_valid, int mode,
     }
     return;
   }
-  /* split Loop Merge (pt_spec<.., NODE, SPLIT>) */
+  /* split Loop Merge (pt_spec<.., NODE, SPLIT>).  WS_SPEC_LOOP_POOL: the warp's
+   * paths form one pool -- path q is sample q / n_valid of the warp's pixel
+   * q % n_valid -- and a lane whose path has ended claims the next unclaimed one
+   * in an advance round, idle lanes in lane order (pt_spec<.., POOL>) */
+  const int pool = mode == WS_SPEC_LOOP_POOL;
+  uint64_t pstart[32 * WS_PT_POOL_MAX_SPP], pend[32 * WS_PT_POOL_MAX_SPP];
+  uint32_t npath = 0, qnext = 0;
+  if (pool) {
+    uint32_t spp = 0;
+    for (uint32_t l = 0; l < n_valid; ++l) {   /* the paths of each lane's pixel */
+      uint32_t k = 0;
+      for (uint64_t i = off[l]; i < off[l + 1]; ++i)
+        if ((ops[i] & 0xE000u) == OR_PT_OP_PATH) k++;
+      if (k > spp) spp = k;
+    }
+    if (spp > WS_PT_POOL_MAX_SPP) spp = WS_PT_POOL_MAX_SPP;
+    for (uint32_t sm = 0; sm < spp; ++sm)      /* pool order: sample-major */
+      for (uint32_t l = 0; l < n_valid; ++l) {
+        uint32_t k = 0;
+        for (uint64_t i = off[l]; i < off[l + 1]; ++i) {
+          if ((ops[i] & 0xE000u) != OR_PT_OP_PATH) continue;
+          if (k++ != sm) continue;
+          uint64_t e = i + 1;
+          while (e < off[l + 1] && (ops[e] & 0xE000u) != OR_PT_OP_PATH) e++;
+          pstart[npath] = i;
+          pend[npath] = e;
+          npath++;
+          break;
+        }
+      }
+    for (uint32_t l = 0; l < 32; ++l) pc[l] = endp[l] = 0;   /* no path held yet */
+  }
   if (T == 0 || T > 32) T = 32;
   uint32_t trav = 0, alive = 0;
-  uint32_t E = ~valid;
-  for (uint32_t l = 0; l < n_valid; ++l) if (pc[l] >= endp[l]) E |= 1u << l;
+  uint32_t E = pool ? 0u : ~valid;   /* with a pool every lane of the warp takes paths */
+  for (uint32_t l = 0; l < n_valid; ++l) if (!pool && pc[l] >= endp[l]) E |= 1u << l;
   for (;;) {
     uint32_t L = 0, I = 0;
     for (uint32_t l = 0; l < 32; ++l) {
@@ -431,6 +463,11 @@ void ws_pt(const uint16_t* ops, const uint64_t* off, uint32_t n_valid, int mode,
         if (ops[pc[l]] & 16u) alive &= ~(1u << l);
         pc[l]++;
       }
+      if (pool && !(alive >> l & 1u) && qnext < npath) {   /* claim the next path */
+        pc[l] = pstart[qnext];
+        endp[l] = pend[qnext];
+        qnext++;
+      }
       if (!(alive >> l & 1u) && pc[l] < endp[l]) {   /* next sample: camera ray */
         pc[l]++;                                     /* the PATH op */
         alive |= 1u << l;
@@ -444,6 +481,6 @@ void ws_pt(const uint16_t* ops, const uint64_t* off, uint32_t n_valid, int mode,
     hit(o, WS_PT_LAUNCH, launch);
     hit(o, WS_PT_TBEGIN, begin);
     for (uint32_t l = 0; l < 32; ++l)
-      if (!(alive >> l & 1u) && pc[l] >= endp[l]) E |= 1u << l;
+      if (!(alive >> l & 1u) && pc[l] >= endp[l] && (!pool || qnext >= npath)) E |= 1u << l;
   }
 }

@@ -7,7 +7,7 @@ import numpy as np
 import pytest
 
 import oracle
-from oracle import PDOM, SPEC_LOOP
+from oracle import PDOM, SPEC_LOOP, SPEC_LOOP_POOL
 from paper_conf_cgo_damanijskymg20_b200 import inputs as I
 from paper_conf_cgo_damanijskymg20_b200 import sr
 
@@ -54,7 +54,7 @@ def test_schedules_replay_every_work_item_once(small, T, U):
         o = off[w:w + 33]
         seg = ops[o[0]:o[-1]]
         nd, lf, sh, pa = _kinds(seg)
-        for mode, t, u in ((PDOM, 0, 1), (SPEC_LOOP, T, U)):
+        for mode, t, u in ((PDOM, 0, 1), (SPEC_LOOP, T, U), (SPEC_LOOP_POOL, T, U)):
             s = oracle.ws_pt(seg, o - o[0], mode, t, u)
             assert s["NODE"][1] == int(nd.sum()) and s["LEAF"][1] == int(lf.sum())
             assert s["SH"][1] == int(sh.sum()) and s["LAUNCH"][1] == int(pa.sum())
@@ -90,3 +90,53 @@ def test_pdom_schedule_closed_form(small):
         rays_per_path.append([int(sh[bounds[i]:bounds[i + 1]].sum()) for i in range(len(starts))])
     rp = np.array(rays_per_path)            # [lane, sample]
     assert s["BOUNCE"][0] == int(rp.max(0).sum()) and s["BOUNCE"][1] == int(rp.sum())
+
+
+@pytest.mark.parametrize("T,U", [(1, 1), (12, 8), (32, 8)])
+def test_pool_reduces_to_fixed_pixels(small, T, U):
+    """the path pool claims path q = (sample q / 32 of pixel q % 32) in lane order:
+    (a) with one sample per pixel the first 32 claims give lane l its own pixel,
+    (b) with 32 identical pixels every lane finishes a sample together with the
+    others and claims its own pixel's next one -- in both cases the schedule is the
+    fixed-pixel one, count for count"""
+    c, ops, off, rgb, ref, rc = small
+    _, _, _, path = _kinds(ops)
+    for w in range(0, c.width * c.height, 32 * 23):
+        o = off[w:w + 33]
+        seg = ops[o[0]:o[-1]]
+        # (a) the first sample of each pixel only
+        lanes = []
+        for l in range(32):
+            lane = ops[off[w + l]:off[w + l + 1]]
+            starts = np.flatnonzero(_kinds(lane)[3])
+            lanes.append(lane[:starts[1]] if len(starts) > 1 else lane)
+        one = np.concatenate(lanes)
+        o1 = np.concatenate([[0], np.cumsum([len(x) for x in lanes])]).astype(np.uint64)
+        assert oracle.ws_pt(one, o1, SPEC_LOOP_POOL, T, U) == oracle.ws_pt(one, o1, SPEC_LOOP, T, U)
+        # (b) 32 copies of pixel w's stream
+        lane0 = ops[off[w]:off[w + 1]]
+        same = np.tile(lane0, 32)
+        o2 = (np.arange(33) * len(lane0)).astype(np.uint64)
+        assert oracle.ws_pt(same, o2, SPEC_LOOP_POOL, T, U) == oracle.ws_pt(same, o2, SPEC_LOOP, T, U)
+
+
+def test_pool_balances_unequal_pixels(small):
+    """a warp whose pixels carry very different work: with the pool the warp needs
+    fewer rounds and its releases run with more lanes (idle lanes take other pixels'
+    samples instead of waiting for the longest pixel)"""
+    c, ops, off, rgb, ref, rc = small
+    # lane l gets pixel w's stream (long) for l < 4, else pixel v's first sample only
+    node, _, _, _ = _kinds(ops)
+    work = np.array([int(node[off[i]:off[i + 1]].sum()) for i in range(len(off) - 1)])
+    w, v = int(np.argmax(work)), int(np.argmin(work))
+    lv = ops[off[v]:off[v + 1]]
+    starts = np.flatnonzero(_kinds(lv)[3])
+    short = lv[:starts[1]] if len(starts) > 1 else lv
+    lanes = [ops[off[w]:off[w + 1]]] * 4 + [short] * 28
+    seg = np.concatenate(lanes)
+    o = np.concatenate([[0], np.cumsum([len(x) for x in lanes])]).astype(np.uint64)
+    fixed = oracle.ws_pt(seg, o, SPEC_LOOP, 12, 8)
+    pooled = oracle.ws_pt(seg, o, SPEC_LOOP_POOL, 12, 8)
+    assert pooled["NODE"][1] == fixed["NODE"][1] and pooled["LEAF"][1] == fixed["LEAF"][1]
+    assert pooled["rounds"] < fixed["rounds"]
+    assert pooled["NODE"][1] / pooled["NODE"][0] > fixed["NODE"][1] / fixed["NODE"][0]
