@@ -620,13 +620,19 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
     c = I.C4
     tris, mat, mats, cam = I.cornell_scene(c)
     buf, used = sr.upload_scene(tris, mat, mats, cam, ctx.device)
-    w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth)
-    ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
+    w_fixed = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth)
+    # the warp's paths pooled (SR_F_POOL): per-path radiance kept for the ordered sums
+    w_pool = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth,
+                                   flags=sr.F_POOL, pool_spp=c.spp)
+    ctx.ensure(sr.sr_workspace_bytes(w_pool, c.n_pixels))
     res = {"scene_triangles": int(len(tris)), "scene_bytes": int(used)}
     # split node-granularity Loop Merge, 8 node visits per release, soft barrier
-    # T = inputs.C4.threshold (best of the threshold sweep, profiles/)
+    # T = inputs.C4.threshold (best of the threshold sweep, profiles/); each lane on
+    # its own pixel, and with the warp's paths pooled
     sname = f"spec_t{c.threshold}"
-    for name, mode, thr in (("pdom", sr.PDOM, 0), (sname, sr.SPEC_LOOP, c.threshold)):
+    for name, mode, thr, w in (("pdom", sr.PDOM, 0, w_fixed),
+                               (sname, sr.SPEC_LOOP, c.threshold, w_fixed),
+                               (sname + "_pool", sr.SPEC_LOOP, c.threshold, w_pool)):
         ms = timer.time_steps(lambda: sr.sr_run(w, c.n_pixels, c.spp, I.PRIMARY_SEED, mode, thr),
                               max(3, min(args.steps, 5)), 1)
         t = statistics.median(ms)
@@ -634,7 +640,9 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
         res[name] = {"value": c.n_pixels * c.spp / (t * 1e-3), "unit": "paths/s", "ms": t,
                      "rays": int(cnt[1]), "node_visits": int(cnt[2]), "tri_tests": int(cnt[3]),
                      "launch": sr.sr_last_launch()}
-    res["speedup_vs_pdom"] = res[sname]["value"] / res["pdom"]["value"]
+    # the merged kernel's best schedule (the pooled paths) and the fixed-pixel one
+    res["speedup_vs_pdom"] = res[sname + "_pool"]["value"] / res["pdom"]["value"]
+    res["speedup_fixed_pixel_vs_pdom"] = res[sname]["value"] / res["pdom"]["value"]
     # issue roofline (as MC): useful work = thread-instructions per path of a PDOM
     # kernel whose lanes each execute only their own path (profiles/work_per_unit.json,
     # pt_basis), peak = 592 SMSPs x 32 lanes x f
@@ -643,7 +651,7 @@ def microbench_configs(torch, sr, I, ctx, stream, timer, args):
         peak = 592 * 32 * f_mhz * 1e6
         res["issue_roofline"] = {
             "thread_inst_per_path": per_path,
-            "frac": {k: per_path * res[k]["value"] / peak for k in ("pdom", sname)},
+            "frac": {k: per_path * res[k]["value"] / peak for k in ("pdom", sname, sname + "_pool")},
             "basis": "profiles/work_per_unit.json pt_thread_inst_per_path (ncu, as-compiled "
                      "PDOM) x paths/s / (592 x 32 x sm_max_mhz)"}
     out["pathtrace"] = res

@@ -92,7 +92,14 @@ typedef enum {
                            iteration) pairs are one queue and every release runs 32 of them,
                            any lane running any thread's call; results are added to each
                            thread's acc in iteration order.  `threshold` is not used.
-                           Results are identical. */
+                           Results are identical.
+                           PATHTRACE + SR_SPEC_LOOP, split node merge (not with COARSE,
+                           NOSPLIT or MATGROUP; needs pathtrace.pool_spp): the warp's
+                           pixels x spp paths form one pool -- a lane whose path has ended
+                           claims the next (sample-major) in an advance round, so no lane
+                           idles while its warp has paths left; each path's radiance is
+                           kept and the pixel sums are formed in sample order at the end.
+                           Images and counters are identical. */
 
 #define SR_MAX_LAYERS 8
 typedef struct { float n, mua, mus, g, d; } sr_layer;  /* -, 1/cm, 1/cm, -, cm */
@@ -151,6 +158,10 @@ typedef struct {
   uint32_t merge_unroll;  /* SR_SPEC_LOOP node-granularity merge: BVH node visits
                              per release round, the partial unroll of P:1467-1474
                              (0 = 8). Results are identical for every value.   */
+  uint32_t pool_spp;      /* with SR_F_POOL: the most samples per pixel (sr_run
+                             iters) a run may ask for, in [1, 4096]; the workspace
+                             then holds 12 * n_threads * pool_spp bytes of per-path
+                             radiance (in SR_T_SCRATCH).  0 without SR_F_POOL.   */
 } sr_pathtrace_params;
 
 typedef struct {
@@ -202,7 +213,7 @@ SR_API int sr_init(int device, void* cuda_stream, void* workspace_dev, size_t wo
  *                   windows x slices (the batched advances), that x valid
  *                   lanes, 0, 0, 0}.  PATHTRACE split merge: words 5, 6 =
  *                   leaf-test releases and their lanes (words 1, 2: node visits)
- *   SR_T_SCRATCH    internal (claim counters)
+ *   SR_T_SCRATCH    internal (claim counters; PATHTRACE + SR_F_POOL: per-path radiance)
  * GRID and COUNTERS are contiguous so a multi-GPU caller can reduce them
  * in place as int64 (two's-complement addition = uint64 addition mod 2^64). */
 enum { SR_T_PERTHREAD = 0, SR_T_GRID = 1, SR_T_COUNTERS = 2, SR_T_SCHED = 3, SR_T_SCRATCH = 4 };

@@ -32,7 +32,7 @@ CC = dict(ENTRY=0, THEN=1, ELSE_PRE=2, CALL=3, ELSE_POST=4, MERGE=5)
 PT = {k: i for i, k in enumerate(
     "ENTRY OUTER LAUNCH BOUNCE TBEGIN STEP NODE PUSH NOPUSH NEXTNONE POP LEAFIF LEAF TT TT_U "
     "TT_V TT_T TT_ID TT_UPD SH SH_HIT SH_SURF SH_DIFF SH_MIRR SH_GLASS SH_RR SH_END ROUND REL "
-    "LREL NREL ADV".split())}
+    "LREL NREL ADV PSUM".split())}
 LM = dict(ENTRY=0, LAUNCH=1, STEP=2, STEP_BOUNDARY=3, STEP_INTERACT=4, ROUND=5, RELEASE=6,
           ADVANCE=7, **{f"EV{b}": 8 + b for b in range(16)}, **{f"NEV{b}": 24 + b for b in range(16)},
           A_RR=40, B_RR=41, B_REL=42, BI=43, A_TAIL=44, CLAIM=45, CLAIMIT=46, CHUNK=47)

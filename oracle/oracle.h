@@ -235,7 +235,8 @@ enum { WS_PT_ENTRY = 0, WS_PT_OUTER, WS_PT_LAUNCH, WS_PT_BOUNCE, WS_PT_TBEGIN, W
        WS_PT_NODE, WS_PT_PUSH, WS_PT_NOPUSH, WS_PT_NEXTNONE, WS_PT_POP, WS_PT_LEAFIF,
        WS_PT_LEAF, WS_PT_TT, WS_PT_TT_U, WS_PT_TT_V, WS_PT_TT_T, WS_PT_TT_ID, WS_PT_TT_UPD,
        WS_PT_SH, WS_PT_SH_HIT, WS_PT_SH_SURF, WS_PT_SH_DIFF, WS_PT_SH_MIRR, WS_PT_SH_GLASS,
-       WS_PT_SH_RR, WS_PT_SH_END, WS_PT_ROUND, WS_PT_REL, WS_PT_LREL, WS_PT_NREL, WS_PT_ADV };
+       WS_PT_SH_RR, WS_PT_SH_END, WS_PT_ROUND, WS_PT_REL, WS_PT_LREL, WS_PT_NREL, WS_PT_ADV,
+       WS_PT_PSUM };
 /* the PDOM (mode WS_PDOM) or split Loop Merge (WS_SPEC_LOOP, threshold T, U
  * work items per release) schedule of one warp of n_valid lanes; WS_SPEC_LOOP_POOL:
  * the split merge with the warp's n_valid x spp paths claimed from one pool

@@ -483,4 +483,7 @@ void ws_pt(const uint16_t* ops, const uint64_t* off, uint32_t n_valid, int mode,
     for (uint32_t l = 0; l < 32; ++l)
       if (!(alive >> l & 1u) && pc[l] >= endp[l] && (!pool || qnext >= npath)) E |= 1u << l;
   }
+  /* with the pool: each valid lane then adds its pixel's samples in sample order */
+  if (pool)
+    for (uint32_t k = 0; k < npath / (n_valid ? n_valid : 1); ++k) hit(o, WS_PT_PSUM, valid);
 }

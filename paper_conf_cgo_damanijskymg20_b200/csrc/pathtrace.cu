@@ -87,6 +87,7 @@ struct PtArgs {
   uint64_t n, seed;
   RoundKeys keys;
   float* rgb;                       // 3 floats per pixel
+  float* prad;                      // POOL: 3 floats per (pixel, sample), pixel-major
   unsigned long long* counters;     // [0] paths [1] rays [2] node visits [3] tri tests
   uint32_t* sched;
   // diagnostics (sr_pt_closest): rays in, hits out
@@ -377,6 +378,9 @@ __device__ __forceinline__ void onb(V3 n, V3& t1, V3& t2) {
 // known (tr finished).  Ends the path when it escaped, hit a light, reached
 // max_depth or lost the roulette; the epilog (pixel sum) happens at that
 // point, in sample order.
+// POOL: a pixel's samples run on several lanes, so each path's radiance is stored
+// at (pixel, sample) and the pixel sum is formed after the warp's pool is done.
+template <bool POOL = false>
 __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
   const int64_t hit = tr.ib;  // @sr-region SH
   const float t = tr.tb;
@@ -437,10 +441,17 @@ __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
   if (end) {
     // Epilog: pixel += radiance, in sample order, in the output itself (a lane owns
     // its pixel; one read-modify-write per path keeps three registers free)
-    float* px = a.rgb + 3 * (uint64_t)p.pix;  // @sr-region SH_END
-    px[0] = px[0] + p.rad.x;
-    px[1] = px[1] + p.rad.y;
-    px[2] = px[2] + p.rad.z;
+    if constexpr (POOL) {
+      float* pr = a.prad + 3 * ((uint64_t)p.pix * a.spp + p.s);  // @sr-region SH_END
+      pr[0] = p.rad.x;
+      pr[1] = p.rad.y;
+      pr[2] = p.rad.z;
+    } else {
+      float* px = a.rgb + 3 * (uint64_t)p.pix;  // @sr-region SH_END
+      px[0] = px[0] + p.rad.x;
+      px[1] = px[1] + p.rad.y;
+      px[2] = px[2] + p.rad.z;
+    }
     p.alive = false;
   }
 }  // @sr-region END
@@ -522,14 +533,21 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_PDOM) pt_pdom(const PtA
 // are grouped by material kind with __match_any_sync; the largest group shades
 // in this advance round (ties: the group of the lowest lane), the others wait
 // in R for a later one.  A miss forms its own group.
-template <bool SCHED, bool NODE, bool SPLIT = false, bool MATG = false>
+// POOL (with SPLIT, SR_F_POOL): the warp's nv pixels x spp samples form one pool of
+// paths, path q = sample q / nv of pixel q % nv; a lane whose path has ended claims
+// the next one in an advance round (idle lanes in lane order), so no lane idles
+// while the warp has paths left -- the fixed-pixel kernel keeps a lane on its own
+// pixel's spp paths and the warp runs until the pixel with the most work is done.
+// Each path's radiance goes to a.prad; the pixel sums are formed at the end in
+// sample order (the same additions as the fixed-pixel epilog).
+template <bool SCHED, bool NODE, bool SPLIT = false, bool MATG = false, bool POOL = false>
 __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtArgs a) {
   const PtHeader& H = *reinterpret_cast<const PtHeader*>(a.scene);  // @sr-region ENTRY:full
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = g < a.n;
   Path p;
   p.pix = (uint32_t)(valid ? g : 0);
-  if (valid) {
+  if (!POOL && valid) {
     float* px = a.rgb + 3 * (uint64_t)p.pix;
     px[0] = 0.0f; px[1] = 0.0f; px[2] = 0.0f;
   }
@@ -539,8 +557,13 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
   bool trav = false;                   // NODE: a ray of this lane is being traversed
   Stats st{0, 0, 0};
   uint32_t paths = 0, rounds = 0, rel = 0, rel_lanes = 0, adv = 0, adv_lanes = 0;
-  uint32_t next_s = 0;
-  uint32_t E = __ballot_sync(kFull, !valid || a.spp == 0);  // lanes with nothing left to do
+  uint32_t next_s = 0;                 // fixed pixel: this lane's next sample; POOL: the
+                                       // warp's next unclaimed path (warp-uniform)
+  // POOL: every lane of the warp takes paths, of the nv valid pixels
+  const uint32_t nv = POOL ? (uint32_t)__popc(__ballot_sync(kFull, valid)) : 0u;
+  const uint32_t pool = nv * a.spp;
+  // lanes with nothing left to do
+  uint32_t E = POOL ? 0u : __ballot_sync(kFull, !valid || a.spp == 0);
   uint32_t lrel = 0, lrel_lanes = 0;
   for (;;) {  // @sr-region ROUND:full
     if constexpr (SPLIT) {
@@ -584,6 +607,27 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
           const uint32_t best = __reduce_max_sync(kFull, score);
           go = go && (!needs || score == best);
         }
+      }
+      if constexpr (POOL) {
+        if (go && p.alive) shade<true>(a, p, tr);  // @sr-region ADV
+        // claims: the lanes of R without a path take the next ones, in lane order
+        const bool need = go && !p.alive;  // @sr-region ADV:full
+        const uint32_t C = __ballot_sync(kFull, need);
+        const uint32_t q = next_s + (uint32_t)__popc(C & lanemask_lt());
+        if (need && q < pool) {
+          p.pix = (uint32_t)(g & ~31ull) + (nv == 32u ? (q & 31u) : q % nv);  // @sr-region LAUNCH
+          p.s = nv == 32u ? (q >> 5) : q / nv;
+          camera_ray(a, H, p);
+          ++paths;
+        }
+        next_s = min(pool, next_s + (uint32_t)__popc(C));  // @sr-region ADV:full
+        if (go && p.alive) {  // @sr-region ADV
+          trav_begin(tr, p.d);  // @sr-region TBEGIN
+          ++st.rays;
+          trav = true;
+        }
+        E = __ballot_sync(kFull, !p.alive && next_s >= pool);  // @sr-region ADV:full
+        continue;
       }
       if (go) {
         if (p.alive) shade(a, p, tr);  // @sr-region ADV
@@ -630,6 +674,22 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
         }
       }
       E = __ballot_sync(kFull, !valid || (!p.alive && next_s >= a.spp));
+    }
+  }
+  if constexpr (POOL) {
+    // the pixel sums, each in sample order, once every path of the warp is done
+    __syncwarp();  // @sr-region ENTRY:full
+    if (valid) {
+      const float* pr = a.prad + 3 * g * a.spp;
+      float r = 0.0f, gg = 0.0f, b = 0.0f;
+#pragma unroll 1  // one sample per trip (the simulator's PSUM count)
+      for (uint32_t s = 0; s < a.spp; ++s) {  // @sr-region PSUM
+        r = r + pr[3 * s];
+        gg = gg + pr[3 * s + 1];
+        b = b + pr[3 * s + 2];
+      }
+      float* px = a.rgb + 3 * g;  // @sr-region ENTRY:full
+      px[0] = r; px[1] = gg; px[2] = b;
     }
   }
   finish(a, p, valid, st, paths, g >> 5, rounds, rel, rel_lanes, adv, adv_lanes, lrel,  // @sr-region ENTRY:full
@@ -751,10 +811,13 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
   a.counters = reinterpret_cast<unsigned long long*>(c.ws + c.lay.off[SR_T_COUNTERS]);
   a.sched = (w.flags & SR_F_SCHED) ? reinterpret_cast<uint32_t*>(c.ws + c.lay.off[SR_T_SCHED])
                                    : nullptr;
+  // POOL: the per-path radiance buffer follows SCRATCH's first 256 bytes (layout_of)
+  a.prad = reinterpret_cast<float*>(c.ws + c.lay.off[SR_T_SCRATCH] + 256);
   const uint32_t block = c.block;
   const uint64_t grid = (n + block - 1) / block;
   if (grid > 0x7fffffffull) return cudaErrorInvalidConfiguration;
   const bool spec = mode == SR_SPEC_LOOP;
+  const bool pool = spec && (w.flags & SR_F_POOL);
   const bool node = (w.flags & SR_F_COARSE) == 0;
   const unsigned gr = (unsigned)grid;
   const size_t smem = (size_t)a.stack_cap * block * sizeof(int32_t);  // traversal stacks
@@ -771,10 +834,15 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
     cudaFuncSetAttribute(pt_spec<true, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaFuncSetAttribute(pt_spec<false, true, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaFuncSetAttribute(pt_spec<true, true, true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<false, true, true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(pt_spec<true, true, true, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   }
   if (!spec) {
     if (a.sched) pt_pdom<true><<<gr, block, smem, c.stream>>>(a);
     else pt_pdom<false><<<gr, block, smem, c.stream>>>(a);
+  } else if (pool) {  // check_pathtrace: split merge only
+    if (a.sched) pt_spec<true, true, true, false, true><<<gr, block, smem, c.stream>>>(a);
+    else pt_spec<false, true, true, false, true><<<gr, block, smem, c.stream>>>(a);
   } else if (node && !(w.flags & SR_F_NOSPLIT) && (w.flags & SR_F_MATGROUP)) {
     if (a.sched) pt_spec<true, true, true, true><<<gr, block, smem, c.stream>>>(a);
     else pt_spec<false, true, true, true><<<gr, block, smem, c.stream>>>(a);

@@ -89,6 +89,13 @@ std::string check_workload(const sr_workload* w, uint64_t n_threads) {
     case SR_WL_MCML:
       return check_mcml(w->mcml);
     case SR_WL_PATHTRACE:
+      if (w->flags & SR_F_POOL) {
+        if (w->flags & (SR_F_COARSE | SR_F_NOSPLIT | SR_F_MATGROUP))
+          return "pathtrace: SR_F_POOL is for the split merge (not with SR_F_COARSE, "
+                 "SR_F_NOSPLIT or SR_F_MATGROUP)";
+        if (w->pathtrace.pool_spp == 0 || w->pathtrace.pool_spp > 4096)
+          return "pathtrace: SR_F_POOL needs pool_spp in [1, 4096]";
+      }
       return check_pathtrace(w->pathtrace, n_threads);
     case SR_WL_RSBENCH:
       if (w->rsbench.fma_count % 8 != 0) return "rsbench.fma_count must be a multiple of 8";
@@ -145,7 +152,11 @@ Layout layout_of(const sr_workload& w, uint64_t n) {
     warps = gw > dyn ? gw : dyn;
   }
   const size_t sched = (w.flags & SR_F_SCHED) ? 4ull * kSchedWords * warps : 0;
-  const size_t bytes[5] = {per, grid, 8ull * kCounters, sched, 256};
+  // SCRATCH: 256 bytes of claim counters, then (PATHTRACE + SR_F_POOL) the per-path
+  // radiance of up to pool_spp samples per pixel, 3 floats each
+  const size_t pool_buf = (w.kind == SR_WL_PATHTRACE && (w.flags & SR_F_POOL))
+                              ? 12ull * n * w.pathtrace.pool_spp : 0;
+  const size_t bytes[5] = {per, grid, 8ull * kCounters, sched, 256 + pool_buf};
   size_t off = 0;
   for (int i = 0; i < 5; ++i) {
     // GRID and COUNTERS adjacent (GRID is a multiple of 8 bytes; no padding
@@ -286,6 +297,9 @@ int sr_run(const sr_workload* w, uint64_t n_threads, uint32_t iters, uint64_t se
   if (mode == SR_SPEC_LOOP && w->kind == SR_WL_COMMONCALL)
     return fail(SR_E_INVALID, "SR_SPEC_LOOP is not valid for SR_WL_COMMONCALL");
   if (threshold > 32) return fail(SR_E_INVALID, "threshold must be in [0, 32]");
+  if (w->kind == SR_WL_PATHTRACE && (w->flags & SR_F_POOL) && iters > w->pathtrace.pool_spp)
+    return fail(SR_E_INVALID, "pathtrace: iters (spp) exceeds pathtrace.pool_spp, the samples "
+                              "per pixel the workspace holds with SR_F_POOL");
   if (mode == SR_SPEC_CALL && threshold != 0 && threshold != 32)
     return fail(SR_E_INVALID, "SR_SPEC_CALL waits for all lanes: threshold must be 0 or 32");
   const uint32_t T = threshold == 0 ? 32u : threshold;
@@ -301,13 +315,14 @@ int sr_run(const sr_workload* w, uint64_t n_threads, uint32_t iters, uint64_t se
   LaunchCtx c{g_ctx.stream, g_ctx.ws, L, g_ctx.sm_count, default_block(*w)};
   cudaError_t e;
   g_launch[3] = 0;
-  // zero the outputs of this run (per-thread outputs are fully overwritten): GRID,
-  // COUNTERS, SCHED and SCRATCH lie back to back (layout_of), so one memset node
-  // covers them and their alignment padding -- one operation per run instead of up
-  // to four keeps the launch overhead of microsecond-scale runs down
+  // zero the outputs of this run (per-thread outputs and the path tracer's per-path
+  // radiance are fully overwritten): GRID, COUNTERS, SCHED and SCRATCH's counters lie
+  // back to back (layout_of), so one memset node covers them and their alignment
+  // padding -- one operation per run instead of up to four keeps the launch overhead
+  // of microsecond-scale runs down
   {
     const size_t z0 = L.off[SR_T_GRID];
-    const size_t z1 = L.off[SR_T_SCRATCH] + L.bytes[SR_T_SCRATCH];
+    const size_t z1 = L.off[SR_T_SCRATCH] + 256;
     if ((e = cudaMemsetAsync(g_ctx.ws + z0, 0, z1 - z0, g_ctx.stream)) != cudaSuccess)
       return fail_cuda(e, "sr_run: cudaMemsetAsync");
   }

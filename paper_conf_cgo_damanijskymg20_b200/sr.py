@@ -62,7 +62,8 @@ class MCMLParams(C.Structure):
 
 class PathtraceParams(C.Structure):
     _fields_ = [("scene_dev", C.c_void_p), ("scene_bytes", C.c_uint64), ("width", C.c_uint32),
-                ("height", C.c_uint32), ("max_depth", C.c_uint32), ("merge_unroll", C.c_uint32)]
+                ("height", C.c_uint32), ("max_depth", C.c_uint32), ("merge_unroll", C.c_uint32),
+                ("pool_spp", C.c_uint32)]
 
 
 class RsbenchParams(C.Structure):
@@ -256,9 +257,11 @@ def upload_scene(tris, mat, mats, cam, device: int = 0):
 
 
 def pathtrace_workload(scene_ptr: int, scene_bytes: int, width: int, height: int, max_depth=8,
-                       flags=0, block=0, unroll=0) -> Workload:
+                       flags=0, block=0, unroll=0, pool_spp=0) -> Workload:
+    """pool_spp: with F_POOL, the most samples per pixel a run may use"""
     w = Workload(kind=WL_PATHTRACE, flags=flags, block_threads=block)
-    w.pathtrace = PathtraceParams(scene_ptr, scene_bytes, width, height, max_depth, unroll)
+    w.pathtrace = PathtraceParams(scene_ptr, scene_bytes, width, height, max_depth, unroll,
+                                  pool_spp)
     return w
 
 

@@ -104,6 +104,12 @@ def test_run_validation_before_state():
     with pytest.raises(sr.SRError) as e:
         sr.sr_run(sr.divloop_workload(batch=64, block=1024), 64, 1, 1, sr.PDOM, 0)
     assert e.value.code == sr.SR_E_INVALID and "block_threads <= 512" in str(e.value)
+    for fl, spp in ((sr.F_POOL, 0), (sr.F_POOL | sr.F_COARSE, 4), (sr.F_POOL | sr.F_MATGROUP, 4),
+                    (sr.F_POOL, 5000)):
+        bad = sr.pathtrace_workload(1 << 20, 1 << 20, 8, 8, flags=fl, pool_spp=spp)
+        with pytest.raises(sr.SRError) as e:
+            sr.sr_run(bad, 64, 4, 1, sr.SPEC_LOOP, 12)
+        assert e.value.code == sr.SR_E_INVALID and "SR_F_POOL" in str(e.value)
     for split in (3, 5, 8):
         bad = sr.divloop_workload(batch=64, flags=sr.F_POOL, split=split)
         with pytest.raises(sr.SRError) as e:

@@ -112,12 +112,18 @@ def test_pool_reduces_to_fixed_pixels(small, T, U):
             lanes.append(lane[:starts[1]] if len(starts) > 1 else lane)
         one = np.concatenate(lanes)
         o1 = np.concatenate([[0], np.cumsum([len(x) for x in lanes])]).astype(np.uint64)
-        assert oracle.ws_pt(one, o1, SPEC_LOOP_POOL, T, U) == oracle.ws_pt(one, o1, SPEC_LOOP, T, U)
+        pooled = oracle.ws_pt(one, o1, SPEC_LOOP_POOL, T, U)
+        assert pooled.pop("PSUM") == (1, 32)        # then one in-order sum per pixel
+        assert pooled == {k: v for k, v in oracle.ws_pt(one, o1, SPEC_LOOP, T, U).items()
+                          if k != "PSUM"}
         # (b) 32 copies of pixel w's stream
         lane0 = ops[off[w]:off[w + 1]]
         same = np.tile(lane0, 32)
         o2 = (np.arange(33) * len(lane0)).astype(np.uint64)
-        assert oracle.ws_pt(same, o2, SPEC_LOOP_POOL, T, U) == oracle.ws_pt(same, o2, SPEC_LOOP, T, U)
+        pooled = oracle.ws_pt(same, o2, SPEC_LOOP_POOL, T, U)
+        assert pooled.pop("PSUM") == (c.spp, 32 * c.spp)
+        assert pooled == {k: v for k, v in oracle.ws_pt(same, o2, SPEC_LOOP, T, U).items()
+                          if k != "PSUM"}
 
 
 def test_pool_balances_unequal_pixels(small):

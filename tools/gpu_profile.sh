@@ -24,6 +24,7 @@ timeout 600 ncu --metrics $M --clock-control none -k regex:divloop --csv --log-f
 timeout 600 ncu --metrics $M --clock-control none -k regex:rs_ --csv --log-file $O/simt_rsstatic_$TAG.csv python tools/one_launch.py rsbench --modes spec --rs-flags 2 > /dev/null 2>&1
 timeout 600 ncu --metrics $M --clock-control none -k regex:divloop --csv --log-file $O/simt_dlpool_$TAG.csv python tools/one_launch.py divloop --dl-batch 64 --dl-flags 32 --modes spec > /dev/null 2>&1
 timeout 600 ncu --metrics $M --clock-control none -k regex:divloop --csv --log-file $O/simt_dlpool4_$TAG.csv python tools/one_launch.py divloop --dl-batch 64 --dl-flags 32 --dl-split 4 --modes spec > /dev/null 2>&1
+timeout 900 ncu --metrics $M --clock-control none -k regex:pt_spec --csv --log-file $O/simt_ptpool_$TAG.csv python tools/one_launch.py pathtrace --modes spec --pt-flags 32 > /dev/null 2>&1
 # the simulator validation launches (static assignment, the oracle replays every warp)
 timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes pdom,spec --threshold 32 --unroll 1 > /dev/null 2>&1
 timeout 600 ncu --metrics $M --clock-control none -k regex:mcml --csv --log-file $O/simt_mcstatic8_$TAG.csv python tools/one_launch.py mcml --static --photons 131072 --iters 8 --modes spec --threshold 8 --unroll 1 > /dev/null 2>&1
@@ -44,10 +45,12 @@ timeout 300 $SC -k regex:divloop_pool -o $O/src_dlpool_$TAG $OL divloop --dl-bat
 timeout 300 $SC -k regex:divloop_pool -o $O/src_dlpool4_$TAG $OL divloop --dl-batch 64 --dl-flags 32 --dl-split 4 --modes spec > /dev/null 2>&1
 timeout 600 $SC -k regex:pt_pdom -o $O/src_pt_pdom_$TAG $OL pathtrace --modes pdom > /dev/null 2>&1
 timeout 600 $SC -k regex:pt_spec -o $O/src_pt_spec_$TAG $OL pathtrace --modes spec > /dev/null 2>&1
+timeout 600 $SC -k regex:pt_spec -o $O/src_pt_pool_$TAG $OL pathtrace --modes spec --pt-flags 32 > /dev/null 2>&1
 # full captures of the path tracer kernels (PDOM and the default split merge)
 # (one kernel per process: a second full capture in the same process came back mostly NaN)
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:pt_pdom -c 1 -o $O/prof_ptpdom_$TAG $OL pathtrace --modes pdom > $O/prof_pt_$TAG.log 2>&1
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:pt_spec -c 1 -o $O/prof_ptspec_$TAG $OL pathtrace --modes spec >> $O/prof_pt_$TAG.log 2>&1
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:pt_spec -c 1 -o $O/prof_ptpool_$TAG $OL pathtrace --modes spec --pt-flags 32 >> $O/prof_pt_$TAG.log 2>&1
 # launch list of one short bench run (shares, not absolutes)
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-cpu --no-configs > $O/launches_$TAG.log 2>&1
 # full captures of the dominant kernel (and its PDOM baseline), at 2M photons

@@ -14,4 +14,5 @@ timeout 900 $S --what rsbench --thresholds $TS --unroll 12 > $O/sweep_rs_$TAG.js
 timeout 900 $S --what rsbench --thresholds $TS --prolog 2048 --unroll 12 > $O/sweep_rsfetch_$TAG.json 2>/dev/null
 timeout 1500 $S --what pathtrace --thresholds $TS --unroll 8 > $O/sweep_pt_$TAG.json 2>/dev/null
 timeout 1500 $S --what pathtrace --thresholds 1,4,8,16,24,32 --flags 4 > $O/sweep_ptcoarse_$TAG.json 2>/dev/null
+timeout 1500 $S --what pathtrace --thresholds $TS --unroll 8 --flags 32 > $O/sweep_ptpool_$TAG.json 2>/dev/null
 ls -la $O/sweep_*_$TAG.json

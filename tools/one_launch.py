@@ -72,7 +72,7 @@ if "pathtrace" in a.what:
     tris, mat, mats, cam = I.cornell_scene(c)
     buf, used = sr.upload_scene(tris, mat, mats, cam)
     w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth,
-                              flags=a.pt_flags)
+                              flags=a.pt_flags, pool_spp=c.spp if a.pt_flags & sr.F_POOL else 0)
     ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
     for md in modes:
         sr.sr_run(w, c.n_pixels, c.spp, seed, sr.PDOM if md == "pdom" else sr.SPEC_LOOP,

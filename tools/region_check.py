@@ -39,7 +39,7 @@ REPORTS = {
     "mcml_pdom_static": "mc_pdom", "mcml_spec_static(T=32)": "mc_spec32",
     "mcml_spec_static(T=8)": "mc_spec8", "mcml_spec_static(T=32,U=4)": "mc_spec32u4",
     "divloop_pool(T=16)": "dlpool", "divloop_pool_split4(T=16)": "dlpool4",
-    "pt_pdom": "pt_pdom", "pt_spec(T=12)": "pt_spec",
+    "pt_pdom": "pt_pdom", "pt_spec(T=12)": "pt_spec", "pt_spec_pool(T=12)": "pt_pool",
 }
 
 

@@ -75,9 +75,10 @@ if "pathtrace" in what:
     tris, mat, mats, cam = I.cornell_scene(c)
     buf, used = sr.upload_scene(tris, mat, mats, cam)
     n = c.width * c.height
-    for flags in (0, sr.F_SCHED, sr.F_NOSPLIT, sr.F_COARSE, sr.F_MATGROUP, sr.F_MATGROUP | sr.F_SCHED):
+    for flags in (0, sr.F_SCHED, sr.F_NOSPLIT, sr.F_COARSE, sr.F_MATGROUP, sr.F_MATGROUP | sr.F_SCHED,
+                  sr.F_POOL, sr.F_POOL | sr.F_SCHED):
         w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth,
-                                  flags=flags)
+                                  flags=flags, pool_spp=2 if flags & sr.F_POOL else 0)
         run(w, n, 2, sr.PDOM, 0)
         for T in (12, 32):
             run(w, n, 2, sr.SPEC_LOOP, T)

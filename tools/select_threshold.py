@@ -82,9 +82,14 @@ def main():
                            lambda mode, T: sp.rsbench_warps(mode, T, pool=True),
                            I.NEXT1.n_threads * I.NEXT1.iters)
     if "pathtrace" in a.what:   # sampled warps (simt_predict.PT_SAMPLE), split merge U = 8
-        fams["pathtrace"] = (r"pt_pdomILb0E", r"pt_specILb0ELb1ELb1ELb0EE",
+        fams["pathtrace"] = (r"pt_pdomILb0E", r"pt_specILb0ELb1ELb1ELb0ELb0EE",
                              lambda mode, T: sp.pt_warps(mode, T, 8),
                              sp.PT_SAMPLE * 32 * I.C4.spp)
+    if "ptpool" in a.what:   # the same with the warp's paths pooled (SR_F_POOL)
+        fams["ptpool"] = (r"pt_pdomILb0E", r"pt_specILb0ELb1ELb1ELb0ELb1EE",
+                          lambda mode, T: sp.pt_warps(
+                              oracle.SPEC_LOOP_POOL if mode == oracle.SPEC_LOOP else mode, T, 8),
+                          sp.PT_SAMPLE * 32 * I.C4.spp)
     if "mcml" in a.what:
         sample = mc_sample(a.mc_warps, a.mc_iters)
         # the PDOM kernel ignores the unroll; SPEC runs U steps per release
@@ -94,9 +99,13 @@ def main():
                         sample[3] * a.mc_iters)
 
     measured = {}
-    for path in a.measured:
+    for path in a.measured:   # FILE, or FAMILY=FILE to file a sweep under another family
+        rename = None
+        if "=" in path:
+            rename, path = path.split("=", 1)
         d = json.load(open(path))
         for fam, rows in d.items():
+            fam = rename or fam
             measured.setdefault(fam, {})
             for r in rows:
                 measured[fam][(r["mode"], r["T"])] = r["ms"]

@@ -228,8 +228,11 @@ CASES = {
     "divloop_pool_split4(T=16)": (r"divloop_pool_splitILi125ELb0ELi4",
                                   lambda: divloop_pool_warps(4)),
     "pt_pdom": (r"pt_pdomILb0E", lambda: pt_warps(oracle.PDOM)),
-    f"pt_spec(T={I.C4.threshold})": (r"pt_specILb0ELb1ELb1ELb0EE",
+    f"pt_spec(T={I.C4.threshold})": (r"pt_specILb0ELb1ELb1ELb0ELb0EE",
                                       lambda: pt_warps(oracle.SPEC_LOOP, I.C4.threshold, 8)),
+    f"pt_spec_pool(T={I.C4.threshold})": (r"pt_specILb0ELb1ELb1ELb0ELb1EE",
+                                           lambda: pt_warps(oracle.SPEC_LOOP_POOL,
+                                                            I.C4.threshold, 8)),
     "mcml_pdom": (r"mcml_pdomILb1ELb0ELb1", lambda: mcml_dyn_warps(oracle.PDOM, 0)),
     "mcml_spec(T=32)": (r"mcml_specILb1ELb0ELb1", lambda: mcml_dyn_warps(oracle.SPEC_LOOP, 32)),
 }

@@ -31,6 +31,7 @@ LABELS_DLBATCH = ["divloop_pdom_batch", "divloop_spec_batch(T=16)"]
 LABELS_RSSTATIC = [f"rs_spec_static(T={_TRS})"]
 LABELS_DLPOOL = ["divloop_pool(T=16)"]
 LABELS_DLPOOL4 = ["divloop_pool_split4(T=16)"]
+LABELS_PTPOOL = [f"pt_spec_pool(T={_I.C4.threshold})"]
 LABELS_MCSTATIC = ["mcml_pdom_static", "mcml_spec_static(T=32)"]
 LABELS_MCSTATIC8 = ["mcml_spec_static(T=8)"]
 LABELS_MCSTATICU4 = ["mcml_spec_static(T=32,U=4)"]
@@ -110,7 +111,8 @@ def main():
                           (f"simt_dlbatch_{tag}.csv", LABELS_DLBATCH),
                           (f"simt_rsstatic_{tag}.csv", LABELS_RSSTATIC),
                           (f"simt_dlpool_{tag}.csv", LABELS_DLPOOL),
-                          (f"simt_dlpool4_{tag}.csv", LABELS_DLPOOL4)):
+                          (f"simt_dlpool4_{tag}.csv", LABELS_DLPOOL4),
+                          (f"simt_ptpool_{tag}.csv", LABELS_PTPOOL)):
         path = os.path.join(OUT, fname)
         if not os.path.exists(path):
             continue

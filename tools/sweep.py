@@ -129,7 +129,8 @@ if "pathtrace" in a.what:
     res = []
     for b in blocks:
         w = sr.pathtrace_workload(buf.data_ptr(), used, c.width, c.height, c.max_depth, block=b,
-                                  flags=a.flags, unroll=a.unroll)
+                                  flags=a.flags, unroll=a.unroll,
+                                  pool_spp=c.spp if a.flags & sr.F_POOL else 0)
         ctx.ensure(sr.sr_workspace_bytes(w, c.n_pixels))
         for mode, T in [(sr.PDOM, 0)] + [(sr.SPEC_LOOP, t) for t in Ts]:
             t = timed(lambda: sr.sr_run(w, c.n_pixels, c.spp, seed, mode, T), a.reps)
