@@ -62,3 +62,6 @@ ls -la $O | tail -30
 timeout 900 python bench.py --photons-per-gpu 1000000000 --steps 3 --warmup 3 --no-configs --no-cpu > $O/bench_c5_$TAG.json 2> $O/bench_c5_$TAG.err
 # CPU baselines of every config, one core and all host cores
 timeout 900 python tools/cpu_baselines.py --out $O/cpu_baselines_$TAG.json > /dev/null 2> $O/cpu_baselines_$TAG.err
+# the reports compress ~5x; gpurun brings back at most 64 MiB (gunzip them here)
+gzip -f $O/*_$TAG.ncu-rep
+du -sh $O
