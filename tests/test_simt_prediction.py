@@ -22,7 +22,7 @@ CASES = ["divloop_pdom", "divloop_spec(T=16)", "divloop_pdom_batch", "divloop_sp
          # the bench's own launches: dynamic photon claiming, U = 4 (sampled warps)
          "mcml_pdom", "mcml_spec(T=32)",
          # configs[3]: the path tracer (sampled warps; oracle.pt_trace work-item streams)
-         "pt_pdom", "pt_spec(T=12)"]
+         "pt_pdom", "pt_spec(T=12)", "pt_spec_pool(T=12)"]
 
 
 @pytest.fixture(scope="module")

@@ -347,13 +347,15 @@ def kernel_costs(kernel_regex=".*"):
         # that step's lanes, so they are costed to the entering region
         regions_here = {f[0] for f in final if f is not None}
         # (the path tracer's PDOM traversal loop is entered once per bounce: BOUNCE)
+        # (the path tracer's split merge: its node releases, NREL -- a simulator count)
         enter = {"STEP": ("BOUNCE" if "BOUNCE" in regions_here else
-                          "RELEASE" if "RELEASE" in regions_here else "LAUNCH"),
+                          "RELEASE" if "RELEASE" in regions_here else
+                          "NREL" if "REL" in regions_here else "LAUNCH"),
                  "PROLOG": "ADVANCE"}
         for rname, ename in enter.items():
             # (ADVANCE has no code of its own when the SCHED counters are compiled
             # out; the simulator still counts its rounds)
-            if ename not in regions_here and ename not in ("LAUNCH", "ADVANCE"):
+            if ename not in regions_here and ename not in ("LAUNCH", "ADVANCE", "NREL"):
                 continue
             idx = [i for i in range(len(body)) if final[i] is not None and final[i][0] == rname
                    and i not in cold]
@@ -361,10 +363,18 @@ def kernel_costs(kernel_regex=".*"):
                 continue
             inner = [(a_, b_) for a_, b_ in loops
                      if sum(a_ <= i <= b_ for i in idx) * 2 > len(idx)]
+            if ename == "NREL":
+                # the split merge's node-release loop is the innermost loop holding most of
+                # the NODE visits; the release's STEP code (loop entry / exit) lies outside it
+                nidx = [i for i in range(len(body)) if final[i] is not None and
+                        final[i][0] == "NODE" and i not in cold]
+                inner = [(a_, b_) for a_, b_ in loops
+                         if sum(a_ <= i <= b_ for i in nidx) * 2 > len(nidx)]
             if ename == "BOUNCE":
-                # the path tracer's PDOM traversal loop: its vote / latch are a few of the
-                # region's instructions, the loop's entry and exit code the rest -- the
-                # innermost loop holding any of them is the traversal loop
+                # the path tracer's PDOM traversal loop (and the split merge's node-release
+                # loop): its vote / latch are a few of the region's instructions, the loop's
+                # entry and exit code the rest -- the innermost loop holding any of them is
+                # the traversal loop
                 inner = [(a_, b_) for a_, b_ in loops if any(a_ <= i <= b_ for i in idx)]
             if not inner:
                 continue
