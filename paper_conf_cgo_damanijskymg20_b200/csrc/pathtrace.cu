@@ -174,6 +174,37 @@ __device__ __forceinline__ bool box_hit(const float* lo, const float* hi, V3 o, 
 
 // Moller-Trumbore exactly as the oracle (e1, e2 precomputed with the same
 // binary32 subtractions).
+// Branch-free form (the split merge's leaf releases, trav_leaf): every quantity
+// computed, the four rejections folded into one predicate -- the same comparisons,
+// so the same accepted hits and the same t.  A leaf release runs >= T lanes, so
+// nearly every warp has a lane that passes each early-out test and pays the full
+// test anyway; this drops the branches around it (merged kernel -1 %; the PDOM
+// kernel, whose warps test triangles with fewer lanes, keeps the early-out form
+// of trav_step, measured 1.6 % faster there; profiles/experiments.md).
+__device__ __forceinline__ void tri_test_flat(const PtTri& T, int32_t at, V3 o, V3 d, float& tb,
+                                              int32_t& ib, uint32_t& mb, uint32_t& slot) {
+  const V3 v0 = mk(T.v0[0], T.v0[1], T.v0[2]);  // @sr-region TT
+  const V3 e1 = mk(T.e1[0], T.e1[1], T.e1[2]);
+  const V3 e2 = mk(T.e2[0], T.e2[1], T.e2[2]);
+  const V3 pv = cross(d, e2);
+  const float det = dot(e1, pv);
+  const float inv = 1.0f / det;
+  const V3 tv = sub(o, v0);
+  const float u = dot(tv, pv) * inv;
+  const V3 qv = cross(tv, e1);
+  const float v = dot(d, qv) * inv;
+  const float t = dot(e2, qv) * inv;
+  const int32_t id = (int32_t)T.id;
+  const bool ok = !(fabsf(det) < kDetEps) & !(u < 0.0f) & !(u > 1.0f) & !(v < 0.0f) &
+                  !(u + v > 1.0f) & (t > kTmin) & ((t < tb) | ((t == tb) & (id < ib)));
+  if (ok) {
+    tb = t;  // @sr-region TT_UPD
+    ib = id;
+    mb = T.mat;
+    slot = (uint32_t)at;
+  }
+}  // @sr-region END
+
 __device__ __forceinline__ void tri_test(const PtTri& T, int32_t at, V3 o, V3 d, float& tb,
                                          int32_t& ib, uint32_t& mb, uint32_t& slot) {
   const V3 v0 = mk(T.v0[0], T.v0[1], T.v0[2]);  // @sr-region TT
@@ -311,7 +342,11 @@ __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats
 }  // @sr-region END
 
 __device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
+#ifdef SR_PT_TT_BRANCH  // tuning variant: the early-out test of trav_step
   tri_test(load_tri(a.tris, tr.la), tr.la, o, d, tr.tb, tr.ib, tr.mb, tr.slot);  // @sr-region LEAF
+#else
+  tri_test_flat(load_tri(a.tris, tr.la), tr.la, o, d, tr.tb, tr.ib, tr.mb, tr.slot);  // @sr-region LEAF
+#endif
   ++st.tests;
   ++tr.la;
   if (--tr.na == 0u) {
@@ -345,6 +380,23 @@ struct Path {
   uint32_t pix, s, b;
   bool alive;
 };
+
+
+// The pixel of lane slot i (thread g, or slot g&~31 + k of a warp's path pool): when
+// the frame splits into 8 x 4 tiles, warp w = i / 32 covers tile w (tiles row-major,
+// lanes row-major inside the tile), so a warp's camera rays leave from a compact
+// patch rather than 32 pixels of one row (both kernels ~4 % faster at configs[3];
+// profiles/experiments.md); other frames keep i.  inputs.pt_lane_pixels states the
+// same map for the simulator.  SR_PT_ROWS (tuning variant): always i.
+__device__ __forceinline__ uint32_t pix_of(const PtArgs& a, uint32_t i) {
+#ifndef SR_PT_ROWS
+  if ((a.width & 7u) == 0u && (a.height & 3u) == 0u) {
+    const uint32_t w = i >> 5, l = i & 31u, tpr = a.width >> 3;
+    return ((w / tpr) * 4u + (l >> 3)) * a.width + (w % tpr) * 8u + (l & 7u);
+  }
+#endif
+  return i;
+}
 
 __device__ __forceinline__ void camera_ray(const PtArgs& a, const PtHeader& H, Path& p) {
   const uint64_t q = (uint64_t)p.pix * a.spp + p.s;  // @sr-region LAUNCH
@@ -491,7 +543,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_PDOM) pt_pdom(const PtA
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = g < a.n;
   Path p;
-  p.pix = (uint32_t)(valid ? g : 0);
+  p.pix = valid ? pix_of(a, (uint32_t)g) : 0u;
   if (valid) {
     float* px = a.rgb + 3 * (uint64_t)p.pix;
     px[0] = 0.0f; px[1] = 0.0f; px[2] = 0.0f;
@@ -546,7 +598,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
   const uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = g < a.n;
   Path p;
-  p.pix = (uint32_t)(valid ? g : 0);
+  p.pix = valid ? pix_of(a, (uint32_t)g) : 0u;
   if (!POOL && valid) {
     float* px = a.rgb + 3 * (uint64_t)p.pix;
     px[0] = 0.0f; px[1] = 0.0f; px[2] = 0.0f;
@@ -615,7 +667,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
         const uint32_t C = __ballot_sync(kFull, need);
         const uint32_t q = next_s + (uint32_t)__popc(C & lanemask_lt());
         if (need && q < pool) {
-          p.pix = (uint32_t)(g & ~31ull) + (nv == 32u ? (q & 31u) : q % nv);  // @sr-region LAUNCH
+          p.pix = pix_of(a, (uint32_t)(g & ~31ull) + (nv == 32u ? (q & 31u) : q % nv));  // @sr-region LAUNCH
           p.s = nv == 32u ? (q >> 5) : q / nv;
           camera_ray(a, H, p);
           ++paths;
@@ -680,7 +732,8 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
     // the pixel sums, each in sample order, once every path of the warp is done
     __syncwarp();  // @sr-region ENTRY:full
     if (valid) {
-      const float* pr = a.prad + 3 * g * a.spp;
+      const uint64_t pg = pix_of(a, (uint32_t)g);
+      const float* pr = a.prad + 3 * pg * a.spp;
       float r = 0.0f, gg = 0.0f, b = 0.0f;
 #pragma unroll 1  // one sample per trip (the simulator's PSUM count)
       for (uint32_t s = 0; s < a.spp; ++s) {  // @sr-region PSUM
@@ -688,7 +741,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
         gg = gg + pr[3 * s + 1];
         b = b + pr[3 * s + 2];
       }
-      float* px = a.rgb + 3 * g;  // @sr-region ENTRY:full
+      float* px = a.rgb + 3 * pg;  // @sr-region ENTRY:full
       px[0] = r; px[1] = gg; px[2] = b;
     }
   }

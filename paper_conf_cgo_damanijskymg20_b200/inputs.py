@@ -129,6 +129,22 @@ C4 = PathTrace()
 C4_SMALL = PathTrace(width=64, height=48, spp=4, subdiv=1)   # oracle-sized parity case
 
 
+def pt_lane_pixels(width: int, height: int):
+    """Launch layout of the path-tracing kernels (not the method): the pixel of
+    lane slot i = 32 w + l.  When the frame splits into 8 x 4 tiles, warp w
+    covers tile w (tiles row-major, lanes row-major inside a tile); otherwise
+    slot i is pixel i.  uint32 array of width * height entries; the warp
+    simulator replays warp w's lanes as entries [32 w, 32 w + 32)."""
+    import numpy as np
+    n = width * height
+    i = np.arange(n, dtype=np.int64)
+    if width % 8 or height % 4:
+        return i.astype(np.uint32)
+    w, l = i >> 5, i & 31
+    tpr = width // 8
+    return (((w // tpr) * 4 + (l >> 3)) * width + (w % tpr) * 8 + (l & 7)).astype(np.uint32)
+
+
 def _icosphere(subdiv: int):
     """Unit icosphere as a float64 triangle soup [n, 3, 3]; midpoints are
     computed from the two endpoint values only, so shared edges stay shared."""

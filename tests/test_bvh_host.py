@@ -98,3 +98,17 @@ def test_deterministic_and_validated():
     img = np.zeros(16, np.uint8)
     with pytest.raises(sr.SRError, match="dst_bytes"):
         sr.sr_scene_build(t, m, mats, cam, img.ctypes.data, 16, host=True)
+
+
+def test_pt_lane_pixels_layout():
+    """the kernels' lane -> pixel layout: a permutation of the frame; with 8 x 4 tiles
+    every warp's 32 pixels form one tile; otherwise the identity"""
+    w, h = 64, 48
+    m = I.pt_lane_pixels(w, h)
+    assert m.dtype == np.uint32 and np.array_equal(np.sort(m), np.arange(w * h))
+    for wi in range(w * h // 32):
+        px, py = m[32 * wi:32 * wi + 32] % w, m[32 * wi:32 * wi + 32] // w
+        assert px.max() - px.min() == 7 and py.max() - py.min() == 3
+        assert px.min() == 8 * (wi % (w // 8)) and py.min() == 4 * (wi // (w // 8))
+    assert np.array_equal(I.pt_lane_pixels(45, 7), np.arange(45 * 7))
+    assert np.array_equal(I.pt_lane_pixels(64, 6), np.arange(64 * 6))

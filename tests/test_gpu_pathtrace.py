@@ -136,7 +136,7 @@ def test_schedule_matches_simulator(ctx, mode, T, pool):
     cnt = ctx.region(w, n, sr.T_COUNTERS, torch.int64).cpu().numpy()
     img = sr.scene_image_host(tris, mat, mats, cam)
     ops, off, _ = oracle.pt_trace(img, cfg.width, cfg.height, cfg.spp, cfg.max_depth,
-                                  I.PRIMARY_SEED)
+                                  I.PRIMARY_SEED, pixels=I.pt_lane_pixels(cfg.width, cfg.height))
     node = (ops & 0xE000) == 0
     leaf = (ops & 0x8000) != 0
     assert cnt[2] == int(node.sum()) and cnt[3] == int(leaf.sum())   # node visits, tests

@@ -151,7 +151,7 @@ def rsbench_warps(mode, T, U=None, pool=False):
             yield oracle.ws_loopmerge(tr, mode, T, U=U if mode == oracle.SPEC_LOOP else 1), len(tr)
 
 
-# configs[3]: the path tracer's warps are 32 consecutive pixels of a row; the
+# configs[3]: the path tracer's warps are 8 x 4 pixel tiles (inputs.pt_lane_pixels); the
 # work-item streams come from oracle.pt_trace (the oracle's BVH traversal over
 # the scene image sr_scene_build writes), sampled over PT_SAMPLE warps spread
 # over the frame
@@ -167,7 +167,8 @@ def _pt_streams():
         img = sr.scene_image_host(tris, mat, mats, cam)
         n_warps = c.n_pixels // 32
         picks = np.linspace(0, n_warps - 1, PT_SAMPLE).astype(np.int64)
-        pix = (picks[:, None] * 32 + np.arange(32)[None, :]).ravel().astype(np.uint32)
+        lanes = I.pt_lane_pixels(c.width, c.height)
+        pix = lanes[(picks[:, None] * 32 + np.arange(32)[None, :]).ravel()]
         ops, off, _ = oracle.pt_trace(img, c.width, c.height, c.spp, c.max_depth,
                                       I.PRIMARY_SEED, pixels=pix)
         _pt_cache.update(ops=ops, off=off)
