@@ -199,7 +199,13 @@ SR_API int sr_init(int device, void* cuda_stream, void* workspace_dev, size_t wo
  *                   DIVLOOP    n_threads x {float acc; uint32 cnt}  (8 B, AoS)
  *                   COMMONCALL n_threads x float y
  *                   MCML       none (0 bytes)
- *                   PATHTRACE  n_threads x float[3] RGB sum over the spp
+ *                   PATHTRACE  n_threads x float[3] RGB sum over the spp, pixel-major
+ *                              (row y, column x at y * width + x).  Lanes to
+ *                              pixels: when width % 8 == 0 and height % 4 == 0,
+ *                              warp w covers the w-th 8 x 4 tile (tiles
+ *                              row-major, lanes row-major inside the tile),
+ *                              else thread g has pixel g; the SR_T_SCHED record
+ *                              of warp w describes that warp's pixels.
  *   SR_T_GRID       MCML: uint64 A[nz][nr], Rd[nr], Tt[nr]  (fixed point, 2^-32)
  *   SR_T_COUNTERS   uint64[16] workload counters (see sr_counter_names in DESIGN.md)
  *   SR_T_SCHED      per warp: uint32[8] schedule counters (only with SR_F_SCHED):
