@@ -35,7 +35,7 @@ typedef struct {
   uint32_t stack_need, pad[3];
 } img_hdr;
 typedef struct {
-  float b0lo[3], b0hi[3], b1lo[3], b1hi[3];
+  float lo[3][2], hi[3][2];   /* [axis][child] */
   int32_t ref0, cnt0, ref1, cnt1;
 } img_node;
 typedef struct {
@@ -127,8 +127,12 @@ static void closest(const unsigned char* img, const img_hdr* H, v3 o, v3 d, hitr
   for (;;) {
     const img_node* N = &nodes[node];
     float tn0 = 0.0f, tn1 = 0.0f;
-    int h0 = N->ref0 >= 0 && box_hit(N->b0lo, N->b0hi, o, inv, h->tb, &tn0);
-    int h1 = N->ref1 >= 0 && box_hit(N->b1lo, N->b1hi, o, inv, h->tb, &tn1);
+    const float lo0[3] = {N->lo[0][0], N->lo[1][0], N->lo[2][0]};
+    const float hi0[3] = {N->hi[0][0], N->hi[1][0], N->hi[2][0]};
+    const float lo1[3] = {N->lo[0][1], N->lo[1][1], N->lo[2][1]};
+    const float hi1[3] = {N->hi[0][1], N->hi[1][1], N->hi[2][1]};
+    int h0 = N->ref0 >= 0 && box_hit(lo0, hi0, o, inv, h->tb, &tn0);
+    int h1 = N->ref1 >= 0 && box_hit(lo1, hi1, o, inv, h->tb, &tn1);
     uint32_t n0 = (h0 && N->cnt0 > 0) ? (uint32_t)N->cnt0 : 0u;
     uint32_t n1 = (h1 && N->cnt1 > 0) ? (uint32_t)N->cnt1 : 0u;
     int in0 = h0 && N->cnt0 == 0, in1 = h1 && N->cnt1 == 0;

@@ -237,18 +237,19 @@ static int build_scene(const char* fn, bool to_device, const float* tris, const 
   }
   std::vector<PtNode> nodes(order.size());
   auto set_child = [&](PtNode& o, int slot, int c) {
-    float* lo = slot ? o.b1lo : o.b0lo;
-    float* hi = slot ? o.b1hi : o.b0hi;
     int32_t& ref = slot ? o.ref1 : o.ref0;
     int32_t& cnt = slot ? o.cnt1 : o.cnt0;
     if (c < 0) {
-      for (int k = 0; k < 3; ++k) { lo[k] = INFINITY; hi[k] = -INFINITY; }
+      for (int k = 0; k < 3; ++k) { o.lo[k][slot] = INFINITY; o.hi[k][slot] = -INFINITY; }
       ref = -1;
       cnt = 0;
       return;
     }
     const BNode& b = B.nodes[c];
-    for (int k = 0; k < 3; ++k) { lo[k] = pad_lo(b.box.lo[k]); hi[k] = pad_hi(b.box.hi[k]); }
+    for (int k = 0; k < 3; ++k) {
+      o.lo[k][slot] = pad_lo(b.box.lo[k]);
+      o.hi[k][slot] = pad_hi(b.box.hi[k]);
+    }
     if (b.count > 0) { ref = b.start; cnt = b.count; }
     else { ref = out_of[c]; cnt = 0; }
   };

@@ -106,31 +106,85 @@ struct Stats {
 // would not vectorise them itself; the image keeps every record 16-byte
 // aligned: 128-byte header, 64-byte nodes, 48-byte triangles).
 // sm_100 has 256-bit global loads: a node (64 bytes, 64-byte aligned in the image)
-// is two LDG.E.256 instead of four LDG.E.128 (SR_PT_LDG128 keeps the latter as a
-// tuning variant).
+// is two LDG.E.256 instead of four LDG.E.128.
 __device__ __forceinline__ void ldg256(const void* p, float4& a, float4& b) {
   asm("ld.global.nc.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
       : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w)
       : "l"(p));
 }
-__device__ __forceinline__ PtNode load_node(const PtNode* base, int32_t i) {
-  const float4* q = reinterpret_cast<const float4*>(base + i);
-#ifdef SR_PT_LDG128
-  const float4 x = __ldg(q), y = __ldg(q + 1), z = __ldg(q + 2);
-  const int4 w = __ldg(reinterpret_cast<const int4*>(q + 3));
+// Conservative slab test against a padded box: accept when the ray's
+// parametric interval [tmin, tbest] can touch the box (slack 1e-5 relative).
+// Callers evaluate it for both child slots unconditionally and AND the result
+// with `slot is not empty` (no branch around the test: the box arithmetic is
+// cheaper than the divergence bookkeeping of a short-circuit).
+#ifdef SR_PT_BOX_BRANCH  // tuning variant: the short-circuit form
+#define SR_PT_SLOT_TEST(REF, HIT) ((REF) >= 0 && (HIT))
 #else
-  float4 x, y, z, wf;
-  ldg256(q, x, y);
-  ldg256(q + 2, z, wf);
-  const int4 w = make_int4(__float_as_int(wf.x), __float_as_int(wf.y), __float_as_int(wf.z),
-                           __float_as_int(wf.w));
+#define SR_PT_SLOT_TEST(REF, HIT) ((HIT) & ((REF) >= 0))
 #endif
-  PtNode n;
-  n.b0lo[0] = x.x; n.b0lo[1] = x.y; n.b0lo[2] = x.z; n.b0hi[0] = x.w;
-  n.b0hi[1] = y.x; n.b0hi[2] = y.y; n.b1lo[0] = y.z; n.b1lo[1] = y.w;
-  n.b1lo[2] = z.x; n.b1hi[0] = z.y; n.b1hi[1] = z.z; n.b1hi[2] = z.w;
-  n.ref0 = w.x; n.cnt0 = w.y; n.ref1 = w.z; n.cnt1 = w.w;
-  return n;
+
+// A node visit's box half: both child boxes against the ray, the slab distances of
+// the two children computed together -- the image interleaves the children per axis
+// (pt_scene.h), so each (lo or hi, axis) is one FADD2 (x - o, o broadcast) and one
+// FMUL2 (* 1/d, broadcast): 12 paired operations instead of 24 scalar ones, the same
+// IEEE roundings.  Then per child the slab interval and the conservative accept test
+// (box_hit's expressions, operand for operand).
+struct NodeVisit {
+  float tn0, tn1;
+  bool h0, h1;        // child slot hit (ANDed with "slot not empty")
+  int32_t ref0, cnt0, ref1, cnt1;
+};
+__device__ __forceinline__ uint64_t fmul2rn(uint64_t a, uint64_t b) {
+  uint64_t d;  // feeds only min / max, so nothing can contract it into an FFMA2
+  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ bool slab_accept(float tx0, float tx1, float ty0, float ty1, float tz0,
+                                            float tz1, float tb, float& tnear) {
+  const float tn = fmaxf(fmaxf(fminf(tx0, tx1), fminf(ty0, ty1)), fmaxf(fminf(tz0, tz1), 0.0f));
+  const float tf = fminf(fminf(fmaxf(tx0, tx1), fmaxf(ty0, ty1)), fmaxf(tz0, tz1));
+  tnear = tn;
+  return tn * (1.0f - 1e-5f) <= tf * (1.0f + 1e-5f) && tn * (1.0f - 1e-5f) <= tb;
+}
+__device__ __forceinline__ NodeVisit visit_node(const PtNode* base, int32_t i, V3 o, V3 inv,
+                                                float tb) {
+  const float4* q = reinterpret_cast<const float4*>(base + i);
+  float4 x, y, z, w;  // x: lo[0][*] lo[1][*]  y: lo[2][*] hi[0][*]  z: hi[1][*] hi[2][*]
+  ldg256(q, x, y);
+  ldg256(q + 2, z, w);
+  const uint64_t nox = pack2(-o.x, -o.x), noy = pack2(-o.y, -o.y), noz = pack2(-o.z, -o.z);
+  const uint64_t ix = pack2(inv.x, inv.x), iy = pack2(inv.y, inv.y), iz = pack2(inv.z, inv.z);
+  float lx0, lx1, ly0, ly1, lz0, lz1, hx0, hx1, hy0, hy1, hz0, hz1;
+  unpack2(fmul2rn(fadd2(pack2(x.x, x.y), nox), ix), lx0, lx1);
+  unpack2(fmul2rn(fadd2(pack2(x.z, x.w), noy), iy), ly0, ly1);
+  unpack2(fmul2rn(fadd2(pack2(y.x, y.y), noz), iz), lz0, lz1);
+  unpack2(fmul2rn(fadd2(pack2(y.z, y.w), nox), ix), hx0, hx1);
+  unpack2(fmul2rn(fadd2(pack2(z.x, z.y), noy), iy), hy0, hy1);
+  unpack2(fmul2rn(fadd2(pack2(z.z, z.w), noz), iz), hz0, hz1);
+  NodeVisit v;
+  v.ref0 = __float_as_int(w.x); v.cnt0 = __float_as_int(w.y);
+  v.ref1 = __float_as_int(w.z); v.cnt1 = __float_as_int(w.w);
+  v.h0 = SR_PT_SLOT_TEST(v.ref0, slab_accept(lx0, hx0, ly0, hy0, lz0, hz0, tb, v.tn0));
+  v.h1 = SR_PT_SLOT_TEST(v.ref1, slab_accept(lx1, hx1, ly1, hy1, lz1, hz1, tb, v.tn1));
+  return v;
+}
+// The same visit with the 24 scalar FADD / FMUL (identical values).
+__device__ __forceinline__ NodeVisit visit_node_scalar(const PtNode* base, int32_t i, V3 o, V3 inv,
+                                                       float tb) {
+  const float4* q = reinterpret_cast<const float4*>(base + i);
+  float4 x, y, z, w;
+  ldg256(q, x, y);
+  ldg256(q + 2, z, w);
+  NodeVisit v;
+  v.ref0 = __float_as_int(w.x); v.cnt0 = __float_as_int(w.y);
+  v.ref1 = __float_as_int(w.z); v.cnt1 = __float_as_int(w.w);
+  v.h0 = SR_PT_SLOT_TEST(v.ref0, slab_accept((x.x - o.x) * inv.x, (y.z - o.x) * inv.x,
+                                             (x.z - o.y) * inv.y, (z.x - o.y) * inv.y,
+                                             (y.x - o.z) * inv.z, (z.z - o.z) * inv.z, tb, v.tn0));
+  v.h1 = SR_PT_SLOT_TEST(v.ref1, slab_accept((x.y - o.x) * inv.x, (y.w - o.x) * inv.x,
+                                             (x.w - o.y) * inv.y, (z.y - o.y) * inv.y,
+                                             (y.y - o.z) * inv.z, (z.w - o.z) * inv.z, tb, v.tn1));
+  return v;
 }
 __device__ __forceinline__ PtTri load_tri(const PtTri* base, int32_t i) {
   const float4* q = reinterpret_cast<const float4*>(base + i);
@@ -151,26 +205,6 @@ __device__ __forceinline__ PtMat load_mat(const PtMat* base, uint32_t i) {
   return m;
 }
 
-// Conservative slab test against a padded box: accept when the ray's
-// parametric interval [tmin, tbest] can touch the box (slack 1e-5 relative).
-// Callers evaluate it for both child slots unconditionally and AND the result
-// with `slot is not empty` (no branch around the test: the box arithmetic is
-// cheaper than the divergence bookkeeping of a short-circuit).
-#ifdef SR_PT_BOX_BRANCH  // tuning variant: the short-circuit form
-#define SR_PT_SLOT_TEST(REF, HIT) ((REF) >= 0 && (HIT))
-#else
-#define SR_PT_SLOT_TEST(REF, HIT) ((HIT) & ((REF) >= 0))
-#endif
-__device__ __forceinline__ bool box_hit(const float* lo, const float* hi, V3 o, V3 inv, float tb,
-                                        float& tnear) {
-  const float tx0 = (lo[0] - o.x) * inv.x, tx1 = (hi[0] - o.x) * inv.x;
-  const float ty0 = (lo[1] - o.y) * inv.y, ty1 = (hi[1] - o.y) * inv.y;
-  const float tz0 = (lo[2] - o.z) * inv.z, tz1 = (hi[2] - o.z) * inv.z;
-  const float tn = fmaxf(fmaxf(fminf(tx0, tx1), fminf(ty0, ty1)), fmaxf(fminf(tz0, tz1), 0.0f));
-  const float tf = fminf(fminf(fmaxf(tx0, tx1), fmaxf(ty0, ty1)), fmaxf(tz0, tz1));
-  tnear = tn;
-  return tn * (1.0f - 1e-5f) <= tf * (1.0f + 1e-5f) && tn * (1.0f - 1e-5f) <= tb;
-}
 
 // Moller-Trumbore exactly as the oracle (e1, e2 precomputed with the same
 // binary32 subtractions).
@@ -274,11 +308,10 @@ __device__ __forceinline__ void trav_begin(Trav& tr, V3 d) {
 
 // returns false when the traversal is finished
 __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
-  const PtNode N = load_node(a.nodes, tr.node);  // @sr-region NODE
+  const NodeVisit N = visit_node(a.nodes, tr.node, o, tr.inv, tr.tb);  // @sr-region NODE
   ++st.nodes;
-  float tn0, tn1;
-  const bool h0 = SR_PT_SLOT_TEST(N.ref0, box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0));
-  const bool h1 = SR_PT_SLOT_TEST(N.ref1, box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1));
+  const float tn0 = N.tn0, tn1 = N.tn1;
+  const bool h0 = N.h0, h1 = N.h1;
   // leaves: test their triangles now (child 0's, then child 1's, one loop);
   // inner children: descend / push
   const int32_t n0 = (h0 && N.cnt0 > 0) ? N.cnt0 : 0, n1 = (h1 && N.cnt1 > 0) ? N.cnt1 : 0;
@@ -313,12 +346,15 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d,
 // the next node exactly as trav_step (node = -1 when the stack is empty).
 // trav_leaf tests ONE queued triangle.  Returns: a leaf triangle is pending
 // (na > 0), else a node is pending (node >= 0), else the traversal is done.
+// PAIRED: the f32x2 box tests (visit_node) or the scalar ones (visit_node_scalar);
+// each kernel takes the form measured faster for it (the path pool: scalar).
+template <bool PAIRED>
 __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats& st) {
-  const PtNode N = load_node(a.nodes, tr.node);  // @sr-region NODE
+  const NodeVisit N = PAIRED ? visit_node(a.nodes, tr.node, o, tr.inv, tr.tb)  // @sr-region NODE
+                             : visit_node_scalar(a.nodes, tr.node, o, tr.inv, tr.tb);
   ++st.nodes;
-  float tn0, tn1;
-  const bool h0 = SR_PT_SLOT_TEST(N.ref0, box_hit(N.b0lo, N.b0hi, o, tr.inv, tr.tb, tn0));
-  const bool h1 = SR_PT_SLOT_TEST(N.ref1, box_hit(N.b1lo, N.b1hi, o, tr.inv, tr.tb, tn1));
+  const float tn0 = N.tn0, tn1 = N.tn1;
+  const bool h0 = N.h0, h1 = N.h1;
   const bool l0 = h0 && N.cnt0 > 0, l1 = h1 && N.cnt1 > 0;
   tr.la = l0 ? N.ref0 : N.ref1;
   tr.na = l0 ? (uint32_t)N.cnt0 : (l1 ? (uint32_t)N.cnt1 : 0u);
@@ -640,7 +676,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
             for (uint32_t k = 0; k < a.unroll && tr.na > 0u; ++k) trav_leaf(a, tr, p.o, p.d, st);  // @sr-region LEAF
           } else {
             for (uint32_t k = 0; k < a.unroll && tr.na == 0u && tr.node >= 0; ++k)  // @sr-region STEP
-              trav_node(a, tr, p.o, st);
+              trav_node<!POOL>(a, tr, p.o, st);
           }
           trav = tr.na > 0u || tr.node >= 0;  // @sr-region REL
         }

@@ -4,7 +4,7 @@
 //   [PtHeader][PtNode x n_nodes][PtTri x n_tris][PtMat x n_mats]
 //
 // PtNode holds BOTH children's boxes (one 64-byte line per visit, the
-// two-wide layout of Aila & Laine): child ref >= 0 with count 0 = inner node
+// two-wide layout of Aila & Laine; the boxes interleaved per axis): child ref >= 0 with count 0 = inner node
 // index; count > 0 = leaf of `count` triangles starting at `ref`; count 0 and
 // ref < 0 = empty slot.  Triangles are stored in BVH order with the edge
 // vectors precomputed (e1 = v1 - v0, e2 = v2 - v0, binary32, the same two
@@ -26,8 +26,10 @@ struct PtHeader {
 };
 static_assert(sizeof(PtHeader) == 128, "PtHeader layout");
 
+// lo[a][c] / hi[a][c]: child c's box on axis a -- the two children interleaved per
+// axis, so one f32x2 operation computes an axis' slab distance for both children
 struct PtNode {
-  float b0lo[3], b0hi[3], b1lo[3], b1hi[3];
+  float lo[3][2], hi[3][2];
   int32_t ref0, cnt0, ref1, cnt1;
 };
 static_assert(sizeof(PtNode) == 64, "PtNode layout");

@@ -13,7 +13,7 @@ from paper_conf_cgo_damanijskymg20_b200 import sr
 HDR = np.dtype([("magic", "<u4"), ("n_nodes", "<u4"), ("n_tris", "<u4"), ("n_mats", "<u4"),
                 ("off_nodes", "<u8"), ("off_tris", "<u8"), ("off_mats", "<u8"), ("bytes", "<u8"),
                 ("cam", "<f4", 16), ("stack_need", "<u4"), ("pad", "<u4", 3)])
-NODE = np.dtype([("b0lo", "<f4", 3), ("b0hi", "<f4", 3), ("b1lo", "<f4", 3), ("b1hi", "<f4", 3),
+NODE = np.dtype([("lo", "<f4", (3, 2)), ("hi", "<f4", (3, 2)),   # [axis][child]
                  ("ref0", "<i4"), ("cnt0", "<i4"), ("ref1", "<i4"), ("cnt1", "<i4")])
 TRI = np.dtype([("v0", "<f4", 3), ("e1", "<f4", 3), ("e2", "<f4", 3), ("id", "<u4"),
                 ("mat", "<u4"), ("pad", "<u4")])
@@ -60,8 +60,8 @@ def test_tree_covers_every_triangle_once_and_boxes_enclose(scene):
         i, d = stack.pop()
         depth_need = max(depth_need, d)
         nd = nodes[i]
-        inner = [(nd["ref0"], nd["cnt0"], nd["b0lo"], nd["b0hi"]),
-                 (nd["ref1"], nd["cnt1"], nd["b1lo"], nd["b1hi"])]
+        inner = [(nd["ref0"], nd["cnt0"], nd["lo"][:, 0], nd["hi"][:, 0]),
+                 (nd["ref1"], nd["cnt1"], nd["lo"][:, 1], nd["hi"][:, 1])]
         both = all(r >= 0 and c == 0 for r, c, _, _ in inner)
         for r, c, lo, hi in inner:
             if r < 0:
@@ -73,9 +73,9 @@ def test_tree_covers_every_triangle_once_and_boxes_enclose(scene):
             else:
                 assert 0 < r < len(nodes)  # pre-order: children after the parent
                 ch = nodes[r]
-                for k in ("b0", "b1"):     # a child's boxes lie inside its parent's box
-                    if ch["ref" + k[1]] >= 0:
-                        assert np.all(ch[k + "lo"] >= lo) and np.all(ch[k + "hi"] <= hi)
+                for k in (0, 1):           # a child's boxes lie inside its parent's box
+                    if ch[f"ref{k}"] >= 0:
+                        assert np.all(ch["lo"][:, k] >= lo) and np.all(ch["hi"][:, k] <= hi)
                 stack.append((r, d + (1 if both else 0)))
     assert np.all(seen == 1)
     assert h["stack_need"] == depth_need

@@ -29,7 +29,6 @@ VARIANTS = {
     "libsr_pt8.so": ["SR_PT_MINB_SPEC=8", "SR_PT_MINB_PDOM=8"],
     "libsr_pt7.so": ["SR_PT_MINB_SPEC=7", "SR_PT_MINB_PDOM=7"],
     "libsr_ptbb.so": ["SR_PT_BOX_BRANCH"],
-    "libsr_pt128.so": ["SR_PT_LDG128"],
     "libsr_ptrows.so": ["SR_PT_ROWS"],
     "libsr_ptttb.so": ["SR_PT_TT_BRANCH"],
 }
