@@ -347,7 +347,13 @@ __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d,
 // trav_leaf tests ONE queued triangle.  Returns: a leaf triangle is pending
 // (na > 0), else a node is pending (node >= 0), else the traversal is done.
 // PAIRED: the f32x2 box tests (visit_node) or the scalar ones (visit_node_scalar);
-// each kernel takes the form measured faster for it (the path pool: scalar).
+// each kernel takes the form measured faster for it (the path pool: scalar;
+// SR_PT_POOL_PAIRED, a tuning variant, gives it the paired form too).
+#ifdef SR_PT_POOL_PAIRED
+constexpr bool kPairedAlways = true;
+#else
+constexpr bool kPairedAlways = false;
+#endif
 template <bool PAIRED>
 __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats& st) {
   const NodeVisit N = PAIRED ? visit_node(a.nodes, tr.node, o, tr.inv, tr.tb)  // @sr-region NODE
@@ -676,7 +682,7 @@ __global__ void __launch_bounds__(SR_PT_MAXT, SR_PT_MINB_SPEC) pt_spec(const PtA
             for (uint32_t k = 0; k < a.unroll && tr.na > 0u; ++k) trav_leaf(a, tr, p.o, p.d, st);  // @sr-region LEAF
           } else {
             for (uint32_t k = 0; k < a.unroll && tr.na == 0u && tr.node >= 0; ++k)  // @sr-region STEP
-              trav_node<!POOL>(a, tr, p.o, st);
+              trav_node<kPairedAlways || !POOL>(a, tr, p.o, st);
           }
           trav = tr.na > 0u || tr.node >= 0;  // @sr-region REL
         }

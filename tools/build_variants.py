@@ -19,7 +19,6 @@ VARIANTS = {
     "libsr_t480m3.so": ["SR_MCML_MAXT=480", "SR_MCML_MINB=3"],
     "libsr_pts5.so": ["SR_PT_MINB_SPEC=5"],
     "libsr_pts7.so": ["SR_PT_MINB_SPEC=7"],
-    "libsr_pts8.so": ["SR_PT_MINB_SPEC=8"],
     "libsr_ptp6.so": ["SR_PT_MINB_PDOM=6"],
     "libsr_ch16.so": ["SR_MC_CHUNK=16"],
     "libsr_ch32.so": ["SR_MC_CHUNK=32"],
@@ -31,6 +30,9 @@ VARIANTS = {
     "libsr_ptbb.so": ["SR_PT_BOX_BRANCH"],
     "libsr_ptrows.so": ["SR_PT_ROWS"],
     "libsr_ptttb.so": ["SR_PT_TT_BRANCH"],
+    "libsr_ptpp8.so": ["SR_PT_POOL_PAIRED", "SR_PT_MINB_SPEC=8"],
+    "libsr_pts8.so": ["SR_PT_MINB_SPEC=8"],
+    "libsr_ptpp.so": ["SR_PT_POOL_PAIRED"],
 }
 if __name__ == "__main__":
     names = sys.argv[1:] or list(VARIANTS)

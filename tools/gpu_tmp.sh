@@ -1,10 +1,9 @@
-# scratch launcher for the current gpurun experiment: profile + the path-tracer sweeps
-TAG=${1:-r02n}
-bash tools/gpu_profile.sh $TAG
+# scratch launcher for the current gpurun experiment (see profiles/experiments.md)
+python -c "import __graft_entry__ as g; g.build()"
 O=gpurun_out
-S="python tools/sweep.py --reps 3"
-TS=1,2,4,8,12,16,20,24,32
-timeout 1500 $S --what pathtrace --thresholds $TS --unroll 8 > $O/sweep_pt_$TAG.json 2>/dev/null
-timeout 1500 $S --what pathtrace --thresholds 1,4,8,16,24,32 --flags 4 > $O/sweep_ptcoarse_$TAG.json 2>/dev/null
-timeout 1500 $S --what pathtrace --thresholds $TS --unroll 8 --flags 32 > $O/sweep_ptpool_$TAG.json 2>/dev/null
-ls -la $O/sweep_*_$TAG.json
+for L in libsr.so libsr_ptpp.so libsr_ptpp8.so libsr_pts8.so libsr.so libsr_ptpp.so libsr_ptpp8.so libsr_pts8.so; do
+  SR_LIB=$PWD/paper_conf_cgo_damanijskymg20_b200/$L timeout 600 python tools/sweep.py --what pathtrace --thresholds 12 --unroll 8 --reps 7 --flags 32 > $O/sw_h_$L.json 2>/dev/null
+  python -c "
+import json;d=json.load(open('$O/sw_h_$L.json'))['pathtrace']
+print('$L pool', [(r['mode'],r['T'],round(r['ms'],2)) for r in d])"
+done

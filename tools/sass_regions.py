@@ -291,6 +291,8 @@ def kernel_costs(kernel_regex=".*"):
                 start = i + 1
         if start < len(body):
             bbs.append((start, len(body)))
+        nested = {i for a, b in loops for i in range(a, b + 1)
+                  if any(a2 < a and b <= b2 or a2 <= a and b < b2 for a2, b2 in loops)}
         final, prev = [None] * len(body), None
         for a_, b_ in bbs:
             # predicated instructions are if-converted branch bodies: they say
@@ -298,6 +300,14 @@ def kernel_costs(kernel_regex=".*"):
             # only unpredicated instructions vote (unless there are none)
             votes, pvotes = {}, {}
             for i in range(a_, b_):
+                # an entry-line special-register read or constant load inside a
+                # nested loop is a rematerialisation (threadIdx, blockDim reloaded
+                # where it is used, e.g. the path tracer's stack address in its
+                # node-release loop): it says nothing about which region the block is in
+                if strong[i] is not None and strong[i][0] == "ENTRY" and \
+                        re.match(r"(S2R|S2UR|CS2R|LDC|LDCU|ULDC)\b", body[i]["text"]) and \
+                        i in nested:
+                    continue
                 if strong[i] is not None and i not in cold:
                     d = pvotes if body[i]["text"].startswith("@") else votes
                     d[strong[i]] = d.get(strong[i], 0) + 1
