@@ -1,10 +1,7 @@
-# scratch launcher for the current gpurun experiment (see profiles/experiments.md)
+# scratch launcher: the driver's round-end checks on the current tree
 python -c "import __graft_entry__ as g; g.build()"
 O=gpurun_out
-for L in libsr.so libsr_ptl2.so libsr_ptpp8.so libsr.so libsr_ptl2.so libsr_ptpp8.so libsr.so libsr_ptl2.so libsr_ptpp8.so; do
-  SR_LIB=$PWD/paper_conf_cgo_damanijskymg20_b200/$L timeout 600 python tools/sweep.py --what pathtrace --thresholds 12 --unroll 8 --reps 7 --flags 32 > $O/sw_i_$L.json 2>/dev/null
-  python -c "
-import json;d=json.load(open('$O/sw_i_$L.json'))['pathtrace']
-print('$L pool', [(r['mode'],r['T'],round(r['ms'],2)) for r in d])"
-done
-SR_LIB=$PWD/paper_conf_cgo_damanijskymg20_b200/libsr_ptl2.so timeout 600 ncu --metrics lts__t_sector_hit_rate.pct,dram__bytes_read.sum,gpu__time_duration.sum --clock-control none -k regex:pt_ --csv python tools/one_launch.py pathtrace --modes pdom,spec --pt-flags 32 2>/dev/null | grep -E "pt_" | cut -c1-250
+timeout 1500 python -m pytest tests -m gpu -x -q > $O/final_tests.log 2>&1; tail -3 $O/final_tests.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/final_smoke.log 2>&1; tail -1 $O/final_smoke.log
+timeout 900 python bench.py > $O/final_bench.json 2> $O/final_bench.err; tail -c 400 $O/final_bench.json
+timeout 900 python bench.py --impl reference --steps 3 --warmup 3 > $O/final_ref.json 2> $O/final_ref.err; tail -c 300 $O/final_ref.json
