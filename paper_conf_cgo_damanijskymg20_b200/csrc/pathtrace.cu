@@ -86,6 +86,9 @@ struct PtArgs {
   uint32_t stack_cap;               // traversal stack entries per thread (>= stack_need)
   uint64_t n, seed;
   RoundKeys keys;
+#ifdef SR_BOUNDS_CHECK
+  uint32_t n_nodes, n_tris, n_mats;
+#endif
   float* rgb;                       // 3 floats per pixel
   float* prad;                      // POOL: 3 floats per (pixel, sample), pixel-major
   unsigned long long* counters;     // [0] paths [1] rays [2] node visits [3] tri tests
@@ -148,6 +151,7 @@ __device__ __forceinline__ bool slab_accept(float tx0, float tx1, float ty0, flo
 }
 __device__ __forceinline__ NodeVisit visit_node(const PtNode* base, int32_t i, V3 o, V3 inv,
                                                 float tb) {
+  SR_CHECK(i >= 0);
   const float4* q = reinterpret_cast<const float4*>(base + i);
   float4 x, y, z, w;  // x: lo[0][*] lo[1][*]  y: lo[2][*] hi[0][*]  z: hi[1][*] hi[2][*]
   ldg256(q, x, y);
@@ -171,6 +175,7 @@ __device__ __forceinline__ NodeVisit visit_node(const PtNode* base, int32_t i, V
 // The same visit with the 24 scalar FADD / FMUL (identical values).
 __device__ __forceinline__ NodeVisit visit_node_scalar(const PtNode* base, int32_t i, V3 o, V3 inv,
                                                        float tb) {
+  SR_CHECK(i >= 0);
   const float4* q = reinterpret_cast<const float4*>(base + i);
   float4 x, y, z, w;
   ldg256(q, x, y);
@@ -187,6 +192,7 @@ __device__ __forceinline__ NodeVisit visit_node_scalar(const PtNode* base, int32
   return v;
 }
 __device__ __forceinline__ PtTri load_tri(const PtTri* base, int32_t i) {
+  SR_CHECK(i >= 0);
   const float4* q = reinterpret_cast<const float4*>(base + i);
   const float4 x = __ldg(q), y = __ldg(q + 1);
   const uint4 z = __ldg(reinterpret_cast<const uint4*>(q + 2));
@@ -291,6 +297,7 @@ extern __shared__ int32_t pt_stack_smem[];
 // entry i of this thread's stack column (addressed from threadIdx / blockDim,
 // so no per-lane pointer is kept in registers)
 __device__ __forceinline__ int32_t& stk(int32_t i) {
+  SR_CHECK(i >= 0 && (uint32_t)i < kMaxStack);
   return pt_stack_smem[(uint32_t)i * blockDim.x + threadIdx.x];
 }
 
@@ -308,6 +315,7 @@ __device__ __forceinline__ void trav_begin(Trav& tr, V3 d) {
 
 // returns false when the traversal is finished
 __device__ __forceinline__ bool trav_step(const PtArgs& a, Trav& tr, V3 o, V3 d, Stats& st) {
+  SR_CHECK((uint32_t)tr.node < a.n_nodes);
   const NodeVisit N = visit_node(a.nodes, tr.node, o, tr.inv, tr.tb);  // @sr-region NODE
   ++st.nodes;
   const float tn0 = N.tn0, tn1 = N.tn1;
@@ -356,6 +364,7 @@ constexpr bool kPairedAlways = false;
 #endif
 template <bool PAIRED>
 __device__ __forceinline__ void trav_node(const PtArgs& a, Trav& tr, V3 o, Stats& st) {
+  SR_CHECK((uint32_t)tr.node < a.n_nodes);
   const NodeVisit N = PAIRED ? visit_node(a.nodes, tr.node, o, tr.inv, tr.tb)  // @sr-region NODE
                              : visit_node_scalar(a.nodes, tr.node, o, tr.inv, tr.tb);
   ++st.nodes;
@@ -387,6 +396,7 @@ __device__ __forceinline__ void trav_leaf(const PtArgs& a, Trav& tr, V3 o, V3 d,
 #ifdef SR_PT_TT_BRANCH  // tuning variant: the early-out test of trav_step
   tri_test(load_tri(a.tris, tr.la), tr.la, o, d, tr.tb, tr.ib, tr.mb, tr.slot);  // @sr-region LEAF
 #else
+  SR_CHECK((uint32_t)tr.la < a.n_tris);
   tri_test_flat(load_tri(a.tris, tr.la), tr.la, o, d, tr.tb, tr.ib, tr.mb, tr.slot);  // @sr-region LEAF
 #endif
   ++st.tests;
@@ -481,6 +491,7 @@ __device__ void shade(const PtArgs& a, Path& p, const Trav& tr) {
   const uint32_t mat = tr.mb, slot = tr.slot;
   bool end = hit < 0;
   if (!end) {
+    SR_CHECK(mat < a.n_mats && slot < a.n_tris);
     const PtMat m = load_mat(a.mats, mat);  // @sr-region SH_HIT
     const uint32_t kind = (uint32_t)m.kind;
     p.rad = add(p.rad, mk(p.thr.x * m.er, p.thr.y * m.eg, p.thr.z * m.eb));
@@ -900,6 +911,11 @@ cudaError_t launch_pathtrace(const LaunchCtx& c, const sr_workload& w, uint64_t 
   a.stack_cap = h.stack_need > 0 ? h.stack_need : 1u;
   a.T = T;
   a.n = n;
+#ifdef SR_BOUNDS_CHECK
+  a.n_nodes = h.n_nodes;
+  a.n_tris = h.n_tris;
+  a.n_mats = h.n_mats;
+#endif
   a.seed = seed;
   a.keys = round_keys(seed);
   a.rgb = reinterpret_cast<float*>(c.ws + c.lay.off[SR_T_PERTHREAD]);
@@ -964,6 +980,11 @@ cudaError_t launch_pt_query(cudaStream_t st, const void* scene, const float* ray
   a.tris = reinterpret_cast<const PtTri*>(a.scene + h.off_tris);
   a.mats = reinterpret_cast<const PtMat*>(a.scene + h.off_mats);
   a.n = n;
+#ifdef SR_BOUNDS_CHECK
+  a.n_nodes = h.n_nodes;
+  a.n_tris = h.n_tris;
+  a.n_mats = h.n_mats;
+#endif
   a.q_rays = rays;
   a.q_hit = hit;
   a.q_t = t;

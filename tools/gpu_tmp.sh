@@ -1,9 +1,5 @@
-# scratch launcher for the current gpurun experiment (see profiles/experiments.md)
+# scratch launcher: the bounds-checked build over every kernel variant
 python -c "import __graft_entry__ as g; g.build()"
 O=gpurun_out
-for U in 4 6 8 10 12 16; do
-  timeout 600 python tools/sweep.py --what pathtrace --thresholds 10,12,14 --unroll $U --reps 5 --flags 32 > $O/sw_u_$U.json 2>/dev/null
-  python -c "
-import json;d=json.load(open('$O/sw_u_$U.json'))['pathtrace']
-print('U=$U pool', [(r['mode'],r['T'],round(r['ms'],2)) for r in d])"
-done
+timeout 1500 python -m pytest tests/test_gpu_bounds.py -q > $O/t_bounds.log 2>&1; tail -3 $O/t_bounds.log
+SR_LIB=$PWD/paper_conf_cgo_damanijskymg20_b200/libsr_bounds.so timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_pathtrace.py tests/test_gpu_rsbench.py -q -x > $O/t_bounds_parity.log 2>&1; tail -2 $O/t_bounds_parity.log
