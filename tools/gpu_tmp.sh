@@ -1,5 +1,6 @@
-# scratch launcher: the bounds-checked build over every kernel variant
+# scratch launcher: the driver's round-end checks on the current tree
 python -c "import __graft_entry__ as g; g.build()"
 O=gpurun_out
-timeout 1500 python -m pytest tests/test_gpu_bounds.py -q > $O/t_bounds.log 2>&1; tail -3 $O/t_bounds.log
-SR_LIB=$PWD/paper_conf_cgo_damanijskymg20_b200/libsr_bounds.so timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_pathtrace.py tests/test_gpu_rsbench.py -q -x > $O/t_bounds_parity.log 2>&1; tail -2 $O/t_bounds_parity.log
+timeout 1500 python -m pytest tests -m gpu -x -q > $O/final2_tests.log 2>&1; tail -3 $O/final2_tests.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/final2_smoke.log 2>&1; tail -1 $O/final2_smoke.log
+timeout 900 python bench.py --steps 5 --warmup 3 > $O/final2_bench.json 2> $O/final2_bench.err; tail -c 200 $O/final2_bench.json
