@@ -1,4 +1,4 @@
-# scratch launcher: the driver's round-end checks on the current tree
+# Run under gpurun: the driver's round-end checks on the current tree (GPU tests incl. the bounds-checked build, smoke, one bench line)
 python -c "import __graft_entry__ as g; g.build()"
 O=gpurun_out
 timeout 1500 python -m pytest tests -m gpu -x -q > $O/final2_tests.log 2>&1; tail -3 $O/final2_tests.log
